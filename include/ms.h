@@ -1,0 +1,165 @@
+/*
+ * ms.h -- C ABI of the B200-native stable multisplit (libms.so).
+ *
+ * Multisplit (§3.1): a permutation of n 32-bit keys, or
+ * key-value pairs, into m contiguous buckets in ascending bucket-id order;
+ * this library is always STABLE (input order kept inside a bucket,
+ * P:358-363), so the output is unique and is defined by Eq. (1) (§4,
+ * P:565-586):  p(i) = sum_{k<j} h_k + |{u_r in B_j : r < i}|  for u_i in B_j.
+ * Optionally the start of every bucket is returned; this library
+ * returns m+1 offsets (the last one is n).
+ *
+ * The hot path is the paper's {pre-scan, scan, post-scan} (§4 P:538-550,
+ * Alg. 1) on tiles of T keys (subproblems of Eq. (2)):
+ *   K1 pre-scan   per-tile bucket histograms H (m x L, bucket-major)
+ *   K2 scan       G = exclusive scan of row-vectorised H, offsets = G[:,0]
+ *   K3 post-scan  recompute ids, stable tile-local multisplit in shared
+ *                 memory, coalesced scatter to G[j][l] + local offset
+ * or the one-pass variant (global histogram + decoupled look-back).
+ *
+ * Conventions for every call below:
+ *  - Pointers named *_in/*_out/ids/offsets/workspace/H/G are CUDA DEVICE
+ *    pointers unless the function name ends in _host.  They must be 16-byte
+ *    aligned (MS_ERR_ALIGNMENT otherwise).  Sizes are element counts.
+ *  - Ownership: the caller owns every buffer; a plan owns only host metadata.
+ *    Nothing here allocates device memory or synchronises, except
+ *    ms_plan_check (synchronises `stream`).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    All work is enqueued on it; results are valid when it completes.
+ *  - Argument errors are returned synchronously before anything is enqueued.
+ *    CUDA launch failures return MS_ERR_CUDA.
+ *  - Out-of-place only: keys_out must not overlap keys_in.
+ */
+#ifndef MS_H
+#define MS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t ms_status;
+#define MS_OK                 0
+#define MS_ERR_INVALID_ARG   (-1) /* null pointer, m out of 1..256, bad kind, n > max_n, ... */
+#define MS_ERR_UNSUPPORTED   (-2) /* e.g. values requested on a key-only plan                 */
+#define MS_ERR_ALIGNMENT     (-3) /* a device pointer is not 16-byte aligned                   */
+#define MS_ERR_ALIAS         (-4) /* an output overlaps an input                               */
+#define MS_ERR_WORKSPACE     (-5) /* workspace NULL or smaller than ms_plan_workspace_size()   */
+#define MS_ERR_CUDA          (-6) /* a CUDA runtime call failed                                */
+#define MS_ERR_BUCKET_RANGE  (-8) /* MS_VALIDATE: some precomputed id was >= m                 */
+
+/* Bucket identifier kinds: the programmer's whatBucket() (P:353-357,
+ * P:810-813) restricted to an enumerated set (readings 7-11). */
+typedef enum {
+  MS_LOWBITS = 0,   /* id = (key >> shift) & (m-1); m must be a power of two            */
+  MS_DELTA = 1,     /* id = min(floor(key / delta), m-1); delta >= 1 (delta-stepping,
+                       P:100-111; the last bucket is the far pile)                       */
+  MS_SPLITTERS = 2, /* id = #{ j : splitters[j] < key } over m-1 non-decreasing splitters
+                       (a key equal to a splitter goes to the lower bucket, Fig. 1(2))    */
+  MS_IDS = 3        /* id = ids[i], precomputed, id_bytes = 1 (u8) or 4 (u32) per id      */
+} ms_bucket_kind;
+
+typedef struct {
+  int32_t kind;               /* ms_bucket_kind                                          */
+  uint32_t m;                 /* number of buckets, 1..256                               */
+  uint32_t shift;             /* MS_LOWBITS: bit offset, shift + log2(m) <= 32           */
+  uint32_t delta;             /* MS_DELTA: bucket width >= 1                             */
+  const uint32_t *splitters;  /* MS_SPLITTERS: HOST pointer to m-1 non-decreasing values,
+                                 copied at ms_plan_create (may be freed afterwards)       */
+  uint32_t id_bytes;          /* MS_IDS: 1 or 4                                          */
+} ms_bucket_spec;
+
+typedef struct ms_plan_s *ms_plan_t;
+
+/* plan flags */
+#define MS_VALIDATE      1u  /* flag precomputed ids >= m on the device; ms_plan_check reports it */
+#define MS_VARIANT_3K    2u  /* force the 3-kernel {pre-scan, scan, post-scan} path              */
+#define MS_VARIANT_1P    4u  /* force the one-pass (histogram + decoupled look-back) path        */
+
+/* Create a plan for up to max_n elements (max_n < 2^32).  with_values != 0
+ * plans key-value runs.  Host-only: validates the spec (m range, power-of-two
+ * m for MS_LOWBITS, delta >= 1, sorted splitters, id_bytes) and precomputes
+ * the bucket-function constants.  Returns MS_ERR_INVALID_ARG on a bad spec. */
+ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n,
+                         int with_values, uint32_t flags);
+
+/* Device workspace bytes ms_run needs for n elements (n <= max_n). */
+ms_status ms_plan_workspace_size(ms_plan_t plan, uint64_t n, size_t *bytes);
+
+/* Tile geometry the plan uses for n elements: tile = T (keys per subproblem),
+ * num_tiles = L = ceil(n / T), variant = 0 (3-kernel) or 1 (one-pass). */
+ms_status ms_plan_geometry(ms_plan_t plan, uint64_t n, uint32_t *tile, uint64_t *num_tiles,
+                           int32_t *variant);
+
+/* The whole multisplit.  keys_in[n] -> keys_out[n]; vals_in/vals_out NULL for
+ * key-only (both non-NULL for key-value); ids[n] (id_bytes each) only for
+ * MS_IDS, else NULL; offsets NULL or m+1 u32 entries (bucket j occupies
+ * [offsets[j], offsets[j+1]), offsets[m] = n).  n = 0 only writes offsets. */
+ms_status ms_run(ms_plan_t plan, const uint32_t *keys_in, const uint32_t *vals_in,
+                 const void *ids, uint32_t *keys_out, uint32_t *vals_out, uint64_t n,
+                 uint32_t *offsets, void *workspace, size_t workspace_bytes, void *stream);
+
+/* ms_run over HOST buffers (pinned for full PCIe rate): copies the inputs to
+ * device staging carved from `workspace`, runs, and copies keys/vals/offsets
+ * back, all on `stream` (host outputs valid once it completes).  Workspace
+ * size: ms_plan_workspace_size_host. */
+ms_status ms_plan_workspace_size_host(ms_plan_t plan, uint64_t n, size_t *bytes);
+ms_status ms_run_host(ms_plan_t plan, const uint32_t *keys_in_host, const uint32_t *vals_in_host,
+                      const void *ids_host, uint32_t *keys_out_host, uint32_t *vals_out_host,
+                      uint64_t n, uint32_t *offsets_host, void *workspace, size_t workspace_bytes,
+                      void *stream);
+
+/* The three stages of the 3-kernel path, individually (for intermediate
+ * parity against Eq. (2); ms_run chains them).  L = ceil(n/T) from
+ * ms_plan_geometry.  H and G are m*L u32, bucket-major (H[j*L + l] = h_{j,l}).
+ *   ms_prescan : H[j][l]  = count of bucket j in tile l         (Alg. 1)
+ *   ms_scan    : G        = exclusive scan of row-vectorised H, in place (H -> G),
+ *                offsets (NULL or m+1) = G[:,0], n              (Alg. 1)
+ *   ms_postscan: keys/vals to G[j][l] + stable local offset     (Alg. 1, §5.2)
+ * `workspace` as for ms_run (ms_plan_workspace_size). */
+ms_status ms_prescan(ms_plan_t plan, const uint32_t *keys_in, const void *ids, uint64_t n,
+                     uint32_t *H, void *workspace, size_t workspace_bytes, void *stream);
+ms_status ms_scan(ms_plan_t plan, uint32_t *HG, uint64_t n, uint32_t *offsets, void *workspace,
+                  size_t workspace_bytes, void *stream);
+ms_status ms_postscan(ms_plan_t plan, const uint32_t *keys_in, const uint32_t *vals_in,
+                      const void *ids, const uint32_t *G, uint32_t *keys_out, uint32_t *vals_out,
+                      uint64_t n, void *workspace, size_t workspace_bytes, void *stream);
+
+/* Device-side whatBucket() only: out_ids[i] = id of keys_in[i] (u32), for
+ * checking the bucket functors (e.g. exhaustively over all 2^32 keys). */
+ms_status ms_bucket_ids(ms_plan_t plan, const uint32_t *keys_in, uint64_t n, uint32_t *out_ids,
+                        void *stream);
+
+/* Synchronises `stream`, then reports MS_ERR_BUCKET_RANGE if a run on this
+ * workspace since the last check saw an id >= m (plans with MS_VALIDATE),
+ * clearing the flag; MS_OK otherwise. */
+ms_status ms_plan_check(ms_plan_t plan, void *workspace, void *stream);
+
+ms_status ms_plan_destroy(ms_plan_t plan);
+const char *ms_status_string(ms_status s);
+
+/* Number of kernel launches the last ms_run / ms_run_host on this plan
+ * enqueued (for the bench's gpu_launches claim). */
+int32_t ms_plan_last_launches(ms_plan_t plan);
+
+/* Per-stage tracing (CUDA events, Table 4's pre-scan / scan /
+ * post-scan split).  ms_plan_trace(plan, 1) clears the record
+ * and makes every following ms_run record an event before its first kernel
+ * and after each kernel on its stream (plan-owned events, created on first
+ * use); ms_plan_trace(plan, 0) stops recording.  ms_plan_trace_read waits
+ * for the recorded events and writes, for up to max_runs runs in order,
+ * stage_ms[r * 4 + s] = duration of stage s of run r in milliseconds
+ * (3-kernel: s = 0 K1, 1 K2, 2 K3; one-pass: 0 histogram, 1 unused (0),
+ * 2 fused pass), and stage_ms[r * 4 + 3] = the run's total; *runs and
+ * *stages (3) report what was written.  Tracing is host-side bookkeeping
+ * only; it adds no kernel launches. */
+ms_status ms_plan_trace(ms_plan_t plan, int enable);
+ms_status ms_plan_trace_read(ms_plan_t plan, float *stage_ms, int32_t max_runs, int32_t *runs,
+                             int32_t *stages);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MS_H */

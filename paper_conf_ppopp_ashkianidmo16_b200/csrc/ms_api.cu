@@ -1,0 +1,507 @@
+// ms_api.cu -- host plan + C ABI of libms.so (see include/ms.h).
+//
+// The plan is host metadata only: validated bucket spec, the bucket-function
+// constants (BucketParams, passed to every kernel by value) and the tile
+// geometry rule.  ms_run enqueues K1 -> K2 -> K3 on the caller's stream with
+// no allocation and no synchronisation.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "../../include/ms.h"
+#include "ms_kernels.cuh"
+
+using namespace ms;
+
+struct ms_plan_s {
+  ms_bucket_spec spec;
+  uint64_t max_n;
+  int kv;
+  uint32_t flags;
+  BucketParams bp;
+  int32_t last_launches;
+  // per-stage trace (ms_plan_trace): one set of 4 events per traced run
+  int tracing = 0;
+  size_t trace_runs = 0;
+  std::vector<cudaEvent_t> trace_ev;  // 4 * capacity
+};
+
+namespace {
+// returns the 4 events for the next traced run (nullptr when not tracing)
+cudaEvent_t *trace_next(ms_plan_s *p) {
+  if (!p->tracing) return nullptr;
+  size_t need = 4 * (p->trace_runs + 1);
+  while (p->trace_ev.size() < need) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+    p->trace_ev.push_back(e);
+  }
+  return &p->trace_ev[4 * p->trace_runs++];
+}
+}  // namespace
+
+namespace {
+
+constexpr size_t kAlign = 256;
+inline size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
+
+uint32_t ceil_log2(uint32_t m) {
+  uint32_t l = 0;
+  while ((1ull << l) < m) ++l;
+  return l;
+}
+
+// Granlund & Montgomery round-up division by an invariant (1 <= d < 2^32):
+// q = (t + ((k - t) >> sh1)) >> sh2,  t = umulhi(k, mul).
+void delta_magic(uint32_t d, uint32_t *mul, uint32_t *sh1, uint32_t *sh2) {
+  uint32_t l = ceil_log2(d);
+  uint64_t num = ((1ull << 32) * ((1ull << l) - d)) / d + 1;  // < 2^32 for d >= 1
+  *mul = (uint32_t)num;
+  *sh1 = l < 1 ? l : 1;
+  *sh2 = l > 0 ? l - 1 : 0;
+}
+
+// Rounds per warp R (tile T = 256 R): 16 for m <= 32, 32 above (runs of T/m
+// keys stay >= 32 keys = 128 B); halved while the grid would not fill two
+// waves of 148 SMs (small n is launch/latency bound, not HBM bound).
+int rounds_for(uint32_t m, uint64_t n) {
+  int R = m <= 32 ? 16 : 32;
+  while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
+  return R;
+}
+
+struct Geometry {
+  int R;
+  uint32_t T;
+  uint64_t L;
+  uint64_t hg_words;   // m * L
+  uint64_t chunks;     // K2 CTAs
+  size_t off_hg, off_status, off_flag, bytes;
+};
+
+Geometry geometry(const ms_plan_s *p, uint64_t n) {
+  Geometry g{};
+  g.R = rounds_for(p->spec.m, n);
+  g.T = 256u * g.R;
+  g.L = (n + g.T - 1) / g.T;
+  g.hg_words = (uint64_t)p->spec.m * g.L;
+  g.chunks = (g.hg_words + kScanChunk - 1) / kScanChunk;
+  // [flag | H/G | look-back status]; the flag sits at offset 0 for every n
+  g.off_flag = 0;
+  g.off_hg = kAlign;
+  g.off_status = g.off_hg + align_up(g.hg_words * 4);
+  g.bytes = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);
+  return g;
+}
+
+bool misaligned(const void *ptr) { return ptr && (reinterpret_cast<uintptr_t>(ptr) & 15u); }
+
+bool overlap(const void *a, size_t abytes, const void *b, size_t bbytes) {
+  if (!a || !b || !abytes || !bbytes) return false;
+  uintptr_t x = (uintptr_t)a, y = (uintptr_t)b;
+  return x < y + bbytes && y < x + abytes;
+}
+
+template <typename K>
+void set_smem(K kernel, size_t bytes) {
+  if (bytes > 48 * 1024) cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+}
+
+size_t k1_smem(uint32_t m) { return (kMaxM + ((m + 3) / 4) * kThreads) * 4; }
+
+size_t k3_smem(int R, bool kv, bool id8) {
+  size_t T = 256u * R;
+  return T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
+}
+
+// ---------------------------------------------------------------- dispatch
+template <int KIND>
+cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const void *ids,
+                      uint32_t n, uint32_t *H, uint64_t *zero_ptr, uint32_t zero_words,
+                      uint32_t *flag, cudaStream_t s) {
+  size_t smem = k1_smem(p->spec.m);
+#define MS_K1(KPT)                                                                         \
+  {                                                                                        \
+    auto k = k1_prescan<KIND, KPT>;                                                        \
+    set_smem(k, smem);                                                                     \
+    k<<<(unsigned)g.L, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, \
+                                            zero_words, flag);                             \
+  }
+  switch (g.R) {
+    case 8: MS_K1(8) break;
+    case 16: MS_K1(16) break;
+    default: MS_K1(32) break;
+  }
+#undef MS_K1
+  return cudaGetLastError();
+}
+
+template <int KIND, bool KV>
+cudaError_t launch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
+                      const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
+                      uint32_t *vo, uint32_t n, cudaStream_t s) {
+  constexpr bool id8 = (KIND == SPLITTERS || KIND == IDS);
+#define MS_K3(R)                                                                             \
+  {                                                                                          \
+    auto k = k3_postscan<KIND, KV, R>;                                                       \
+    size_t smem = k3_smem(R, KV, id8);                                                       \
+    set_smem(k, smem);                                                                       \
+    k<<<(unsigned)g.L, kThreads, smem, s>>>(keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->bp); \
+  }
+  switch (g.R) {
+    case 8: MS_K3(8) break;
+    case 16: MS_K3(16) break;
+    default: MS_K3(32) break;
+  }
+#undef MS_K3
+  return cudaGetLastError();
+}
+
+cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const void *ids,
+                        uint32_t n, uint32_t *H, uint64_t *zp, uint32_t zw, uint32_t *flag,
+                        cudaStream_t s) {
+  switch (p->spec.kind) {
+    case MS_LOWBITS: return launch_k1<LOWBITS>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case MS_DELTA: return launch_k1<DELTA>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case MS_SPLITTERS: return launch_k1<SPLITTERS>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    default: return launch_k1<IDS>(p, g, keys, ids, n, H, zp, zw, flag, s);
+  }
+}
+
+cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
+                        const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
+                        uint32_t *vo, uint32_t n, cudaStream_t s) {
+  const bool kv = vals != nullptr;
+#define MS_K3K(KIND)                                                     \
+  return kv ? launch_k3<KIND, true>(p, g, keys, vals, ids, G, ko, vo, n, s) \
+            : launch_k3<KIND, false>(p, g, keys, vals, ids, G, ko, vo, n, s);
+  switch (p->spec.kind) {
+    case MS_LOWBITS: MS_K3K(LOWBITS)
+    case MS_DELTA: MS_K3K(DELTA)
+    case MS_SPLITTERS: MS_K3K(SPLITTERS)
+    default: MS_K3K(IDS)
+  }
+#undef MS_K3K
+}
+
+ms_status check_ws(const ms_plan_s *p, uint64_t n, void *ws, size_t ws_bytes, Geometry *g) {
+  *g = geometry(p, n);
+  if (!ws || ws_bytes < g->bytes) return MS_ERR_WORKSPACE;
+  if (misaligned(ws)) return MS_ERR_ALIGNMENT;
+  return MS_OK;
+}
+
+ms_status check_common(const ms_plan_s *p, const uint32_t *keys_in, const void *ids, uint64_t n) {
+  if (!p) return MS_ERR_INVALID_ARG;
+  if (n > p->max_n || n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
+  if (n > 0 && !keys_in) return MS_ERR_INVALID_ARG;
+  if (n > 0 && p->spec.kind == MS_IDS && !ids) return MS_ERR_INVALID_ARG;
+  if (misaligned(keys_in) || misaligned(ids)) return MS_ERR_ALIGNMENT;
+  return MS_OK;
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+const char *ms_status_string(ms_status s) {
+  switch (s) {
+    case MS_OK: return "ok";
+    case MS_ERR_INVALID_ARG: return "invalid argument";
+    case MS_ERR_UNSUPPORTED: return "unsupported";
+    case MS_ERR_ALIGNMENT: return "pointer not 16-byte aligned";
+    case MS_ERR_ALIAS: return "output overlaps input";
+    case MS_ERR_WORKSPACE: return "workspace missing or too small";
+    case MS_ERR_CUDA: return "CUDA error";
+    case MS_ERR_BUCKET_RANGE: return "bucket id >= m";
+    default: return "unknown status";
+  }
+}
+
+ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n,
+                         int with_values, uint32_t flags) {
+  if (!plan || !spec) return MS_ERR_INVALID_ARG;
+  *plan = nullptr;
+  const uint32_t m = spec->m;
+  if (m < 1 || m > (uint32_t)kMaxM) return MS_ERR_INVALID_ARG;
+  if (max_n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
+  if ((flags & MS_VARIANT_3K) && (flags & MS_VARIANT_1P)) return MS_ERR_INVALID_ARG;
+  if (flags & ~(MS_VALIDATE | MS_VARIANT_3K | MS_VARIANT_1P)) return MS_ERR_INVALID_ARG;
+  BucketParams bp;
+  memset(&bp, 0, sizeof(bp));
+  bp.m = m;
+  bp.mmask = m - 1;
+  bp.logm = ceil_log2(m);
+  bp.validate = (flags & MS_VALIDATE) ? 1u : 0u;
+  switch (spec->kind) {
+    case MS_LOWBITS:
+      if (m & (m - 1)) return MS_ERR_INVALID_ARG;  // reading #10
+      if (spec->shift > 31 || spec->shift + bp.logm > 32) return MS_ERR_INVALID_ARG;
+      bp.shift = spec->shift;
+      break;
+    case MS_DELTA:
+      if (spec->delta < 1) return MS_ERR_INVALID_ARG;
+      delta_magic(spec->delta, &bp.dmul, &bp.dsh1, &bp.dsh2);
+      break;
+    case MS_SPLITTERS: {
+      if (m > 1 && !spec->splitters) return MS_ERR_INVALID_ARG;
+      for (uint32_t j = 0; j < (1u << bp.logm); ++j) bp.spl[j] = 0xFFFFFFFFu;
+      for (uint32_t j = 0; j + 1 < m; ++j) {
+        if (j > 0 && spec->splitters[j] < spec->splitters[j - 1]) return MS_ERR_INVALID_ARG;
+        bp.spl[j] = spec->splitters[j];
+      }
+      break;
+    }
+    case MS_IDS:
+      if (spec->id_bytes != 1 && spec->id_bytes != 4) return MS_ERR_INVALID_ARG;
+      bp.id_bytes = spec->id_bytes;
+      break;
+    default: return MS_ERR_INVALID_ARG;
+  }
+  ms_plan_s *p = new (std::nothrow) ms_plan_s;
+  if (!p) return MS_ERR_INVALID_ARG;
+  p->spec = *spec;
+  p->spec.splitters = nullptr;  // copied into bp.spl
+  p->max_n = max_n;
+  p->kv = with_values ? 1 : 0;
+  p->flags = flags;
+  p->bp = bp;
+  p->last_launches = 0;
+  *plan = p;
+  return MS_OK;
+}
+
+ms_status ms_plan_destroy(ms_plan_t plan) {
+  if (plan)
+    for (cudaEvent_t e : plan->trace_ev) cudaEventDestroy(e);
+  delete plan;
+  return MS_OK;
+}
+
+ms_status ms_plan_workspace_size(ms_plan_t p, uint64_t n, size_t *bytes) {
+  if (!p || !bytes || n > p->max_n) return MS_ERR_INVALID_ARG;
+  *bytes = geometry(p, n).bytes;
+  return MS_OK;
+}
+
+ms_status ms_plan_geometry(ms_plan_t p, uint64_t n, uint32_t *tile, uint64_t *num_tiles,
+                           int32_t *variant) {
+  if (!p || n > p->max_n) return MS_ERR_INVALID_ARG;
+  Geometry g = geometry(p, n);
+  if (tile) *tile = g.T;
+  if (num_tiles) *num_tiles = g.L;
+  if (variant) *variant = 0;
+  return MS_OK;
+}
+
+int32_t ms_plan_last_launches(ms_plan_t p) { return p ? p->last_launches : -1; }
+
+ms_status ms_plan_trace(ms_plan_t p, int enable) {
+  if (!p) return MS_ERR_INVALID_ARG;
+  if (enable) p->trace_runs = 0;
+  p->tracing = enable ? 1 : 0;
+  return MS_OK;
+}
+
+ms_status ms_plan_trace_read(ms_plan_t p, float *stage_ms, int32_t max_runs, int32_t *runs, int32_t *stages) {
+  if (!p || (!stage_ms && max_runs > 0)) return MS_ERR_INVALID_ARG;
+  int32_t r = (int32_t)std::min<size_t>(p->trace_runs, (size_t)std::max(max_runs, 0));
+  for (int32_t i = 0; i < r; ++i) {
+    cudaEvent_t *ev = &p->trace_ev[4 * i];
+    if (cudaEventSynchronize(ev[3]) != cudaSuccess) return MS_ERR_CUDA;
+    for (int s = 0; s < 3; ++s)
+      if (cudaEventElapsedTime(&stage_ms[4 * i + s], ev[s], ev[s + 1]) != cudaSuccess) return MS_ERR_CUDA;
+    if (cudaEventElapsedTime(&stage_ms[4 * i + 3], ev[0], ev[3]) != cudaSuccess) return MS_ERR_CUDA;
+  }
+  if (runs) *runs = r;
+  if (stages) *stages = 3;
+  return MS_OK;
+}
+
+ms_status ms_prescan(ms_plan_t p, const uint32_t *keys_in, const void *ids, uint64_t n,
+                     uint32_t *H, void *ws, size_t ws_bytes, void *stream) {
+  ms_status st = check_common(p, keys_in, ids, n);
+  if (st != MS_OK) return st;
+  if (!H) return MS_ERR_INVALID_ARG;
+  if (misaligned(H)) return MS_ERR_ALIGNMENT;
+  Geometry g;
+  if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
+  if (n == 0) return MS_OK;
+  char *w = (char *)ws;
+  cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, H, nullptr, 0,
+                              (uint32_t *)(w + g.off_flag), (cudaStream_t)stream);
+  return e == cudaSuccess ? MS_OK : MS_ERR_CUDA;
+}
+
+ms_status ms_scan(ms_plan_t p, uint32_t *HG, uint64_t n, uint32_t *offsets, void *ws,
+                  size_t ws_bytes, void *stream) {
+  if (!p || n > p->max_n) return MS_ERR_INVALID_ARG;
+  if (misaligned(HG) || misaligned(offsets)) return MS_ERR_ALIGNMENT;
+  Geometry g;
+  ms_status st = check_ws(p, n, ws, ws_bytes, &g);
+  if (st != MS_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n == 0) {
+    if (offsets && cudaMemsetAsync(offsets, 0, (p->spec.m + 1) * 4, s) != cudaSuccess) return MS_ERR_CUDA;
+    return MS_OK;
+  }
+  if (!HG) return MS_ERR_INVALID_ARG;
+  char *w = (char *)ws;
+  uint64_t *status = (uint64_t *)(w + g.off_status);
+  if (cudaMemsetAsync(status, 0, g.chunks * 8, s) != cudaSuccess) return MS_ERR_CUDA;
+  k2_scan<<<(unsigned)g.chunks, kThreads, 0, s>>>(HG, g.hg_words, status, offsets, (uint32_t)g.L,
+                                                 p->spec.m, (uint32_t)n);
+  return cudaGetLastError() == cudaSuccess ? MS_OK : MS_ERR_CUDA;
+}
+
+ms_status ms_postscan(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in,
+                      const void *ids, const uint32_t *G, uint32_t *keys_out, uint32_t *vals_out,
+                      uint64_t n, void *ws, size_t ws_bytes, void *stream) {
+  ms_status st = check_common(p, keys_in, ids, n);
+  if (st != MS_OK) return st;
+  if ((vals_in == nullptr) != (vals_out == nullptr)) return MS_ERR_INVALID_ARG;
+  if (vals_in && !p->kv) return MS_ERR_UNSUPPORTED;
+  if (n > 0 && (!G || !keys_out)) return MS_ERR_INVALID_ARG;
+  if (misaligned(vals_in) || misaligned(G) || misaligned(keys_out) || misaligned(vals_out))
+    return MS_ERR_ALIGNMENT;
+  Geometry g;
+  if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
+  if (n == 0) return MS_OK;
+  cudaError_t e = dispatch_k3(p, g, keys_in, vals_in, ids, G, keys_out, vals_out, (uint32_t)n,
+                              (cudaStream_t)stream);
+  return e == cudaSuccess ? MS_OK : MS_ERR_CUDA;
+}
+
+ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, const void *ids,
+                 uint32_t *keys_out, uint32_t *vals_out, uint64_t n, uint32_t *offsets, void *ws,
+                 size_t ws_bytes, void *stream) {
+  ms_status st = check_common(p, keys_in, ids, n);
+  if (st != MS_OK) return st;
+  if ((vals_in == nullptr) != (vals_out == nullptr)) return MS_ERR_INVALID_ARG;
+  if (vals_in && !p->kv) return MS_ERR_UNSUPPORTED;
+  if (n > 0 && !keys_out) return MS_ERR_INVALID_ARG;
+  if (misaligned(vals_in) || misaligned(keys_out) || misaligned(vals_out) || misaligned(offsets))
+    return MS_ERR_ALIGNMENT;
+  const size_t nb = n * 4;
+  if (overlap(keys_out, nb, keys_in, nb) || overlap(keys_out, nb, vals_in, nb) ||
+      overlap(vals_out, nb, keys_in, nb) || overlap(vals_out, nb, vals_in, nb) ||
+      overlap(keys_out, nb, vals_out, nb) ||
+      overlap(keys_out, nb, ids, n * p->spec.id_bytes) || overlap(vals_out, nb, ids, n * p->spec.id_bytes))
+    return MS_ERR_ALIAS;
+  Geometry g;
+  if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  p->last_launches = 0;
+  if (n == 0) {
+    if (offsets && cudaMemsetAsync(offsets, 0, (p->spec.m + 1) * 4, s) != cudaSuccess) return MS_ERR_CUDA;
+    return MS_OK;
+  }
+  char *w = (char *)ws;
+  uint32_t *HG = (uint32_t *)(w + g.off_hg);
+  uint64_t *status = (uint64_t *)(w + g.off_status);
+  uint32_t *flag = (uint32_t *)(w + g.off_flag);
+  if ((p->flags & MS_VALIDATE) && p->spec.kind == MS_IDS &&
+      cudaMemsetAsync(flag, 0, 4, s) != cudaSuccess)
+    return MS_ERR_CUDA;
+  cudaEvent_t *ev = trace_next(p);
+  if (ev) cudaEventRecord(ev[0], s);
+  cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, status, (uint32_t)g.chunks, flag, s);
+  if (e != cudaSuccess) return MS_ERR_CUDA;
+  if (ev) cudaEventRecord(ev[1], s);
+  k2_scan<<<(unsigned)g.chunks, kThreads, 0, s>>>(HG, g.hg_words, status, offsets, (uint32_t)g.L,
+                                                 p->spec.m, (uint32_t)n);
+  if (cudaGetLastError() != cudaSuccess) return MS_ERR_CUDA;
+  if (ev) cudaEventRecord(ev[2], s);
+  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, s);
+  if (e != cudaSuccess) return MS_ERR_CUDA;
+  if (ev) cudaEventRecord(ev[3], s);
+  p->last_launches = 3;
+  return MS_OK;
+}
+
+ms_status ms_plan_workspace_size_host(ms_plan_t p, uint64_t n, size_t *bytes) {
+  if (!p || !bytes || n > p->max_n) return MS_ERR_INVALID_ARG;
+  size_t ws = geometry(p, n).bytes;
+  size_t arr = align_up(n * 4);
+  size_t stage = arr * (p->kv ? 4 : 2) + (p->spec.kind == MS_IDS ? align_up(n * p->spec.id_bytes) : 0) +
+                 align_up((p->spec.m + 1) * 4);
+  *bytes = ws + stage;
+  return MS_OK;
+}
+
+ms_status ms_run_host(ms_plan_t p, const uint32_t *keys_h, const uint32_t *vals_h, const void *ids_h,
+                      uint32_t *keys_out_h, uint32_t *vals_out_h, uint64_t n, uint32_t *offsets_h,
+                      void *ws, size_t ws_bytes, void *stream) {
+  if (!p || n > p->max_n) return MS_ERR_INVALID_ARG;
+  if ((vals_h == nullptr) != (vals_out_h == nullptr)) return MS_ERR_INVALID_ARG;
+  if (vals_h && !p->kv) return MS_ERR_UNSUPPORTED;
+  if (n > 0 && (!keys_out_h || !keys_h || (p->spec.kind == MS_IDS && !ids_h)))
+    return MS_ERR_INVALID_ARG;
+  size_t need = 0;
+  ms_plan_workspace_size_host(p, n, &need);
+  if (!ws || ws_bytes < need) return MS_ERR_WORKSPACE;
+  if (misaligned(ws)) return MS_ERR_ALIGNMENT;
+  cudaStream_t s = (cudaStream_t)stream;
+  Geometry g = geometry(p, n);
+  char *w = (char *)ws + g.bytes;
+  size_t arr = align_up(n * 4);
+  uint32_t *dk = (uint32_t *)w; w += arr;
+  uint32_t *dko = (uint32_t *)w; w += arr;
+  uint32_t *dv = nullptr, *dvo = nullptr;
+  if (p->kv) { dv = (uint32_t *)w; w += arr; dvo = (uint32_t *)w; w += arr; }
+  void *did = nullptr;
+  if (p->spec.kind == MS_IDS) { did = w; w += align_up(n * p->spec.id_bytes); }
+  uint32_t *doff = (uint32_t *)w;
+  if (n > 0) {
+    if (keys_h && cudaMemcpyAsync(dk, keys_h, n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) return MS_ERR_CUDA;
+    if (vals_h && cudaMemcpyAsync(dv, vals_h, n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) return MS_ERR_CUDA;
+    if (did && cudaMemcpyAsync(did, ids_h, n * p->spec.id_bytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
+      return MS_ERR_CUDA;
+  }
+  ms_status st = ms_run(p, keys_h ? dk : nullptr, vals_h ? dv : nullptr, did, dko, vals_h ? dvo : nullptr, n,
+                        offsets_h ? doff : nullptr, ws, g.bytes, stream);
+  if (st != MS_OK) return st;
+  if (n > 0) {
+    if (cudaMemcpyAsync(keys_out_h, dko, n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess) return MS_ERR_CUDA;
+    if (vals_out_h && cudaMemcpyAsync(vals_out_h, dvo, n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+      return MS_ERR_CUDA;
+  }
+  if (offsets_h && cudaMemcpyAsync(offsets_h, doff, (p->spec.m + 1) * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+    return MS_ERR_CUDA;
+  return MS_OK;
+}
+
+ms_status ms_bucket_ids(ms_plan_t p, const uint32_t *keys_in, uint64_t n, uint32_t *out_ids, void *stream) {
+  if (!p || !keys_in || !out_ids) return MS_ERR_INVALID_ARG;
+  if (p->spec.kind == MS_IDS) return MS_ERR_UNSUPPORTED;
+  if (misaligned(keys_in) || misaligned(out_ids)) return MS_ERR_ALIGNMENT;
+  if (n == 0) return MS_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  unsigned grid = (unsigned)std::min<uint64_t>((n + kThreads - 1) / kThreads, 148ull * 16);
+  switch (p->spec.kind) {
+    case MS_LOWBITS: k_bucket_ids<LOWBITS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+    case MS_DELTA: k_bucket_ids<DELTA><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+    default: k_bucket_ids<SPLITTERS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+  }
+  return cudaGetLastError() == cudaSuccess ? MS_OK : MS_ERR_CUDA;
+}
+
+ms_status ms_plan_check(ms_plan_t p, void *ws, void *stream) {
+  if (!p || !ws) return MS_ERR_INVALID_ARG;
+  cudaStream_t s = (cudaStream_t)stream;
+  uint32_t host = 0;
+  if (cudaMemcpyAsync(&host, ws, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess) return MS_ERR_CUDA;
+  if (cudaStreamSynchronize(s) != cudaSuccess) return MS_ERR_CUDA;
+  if (host) {
+    if (cudaMemsetAsync(ws, 0, 4, s) != cudaSuccess) return MS_ERR_CUDA;
+    return MS_ERR_BUCKET_RANGE;
+  }
+  return MS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,158 @@
+// ms_device.cuh -- device primitives of the B200 multisplit (sm_100a).
+//
+// Bucket functors (whatBucket()), warp vote
+// helpers (the ballot/popc machinery of Alg. 2/3, §5.1) and the
+// TMA bulk-copy + mbarrier wrappers used to stage tiles in shared memory.
+#pragma once
+#include <cstdint>
+
+namespace ms {
+
+enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3 };
+
+constexpr int kThreads = 256;  // CTA = 8 warps (the paper's NW = 8)
+constexpr int kWarps = kThreads / 32;
+constexpr int kMaxM = 256;
+
+// Bucket-function constants, passed by value as a kernel parameter (lives in
+// the constant bank; no device allocation).  spl[] holds the splitters padded
+// to Q = 2^logm entries with 0xFFFFFFFF (never "< key"), so the branchless
+// search below always runs exactly logm steps.
+struct BucketParams {
+  uint32_t m;         // number of buckets (1..256)
+  uint32_t mmask;     // m - 1
+  uint32_t shift;     // LOWBITS bit offset
+  uint32_t dmul;      // DELTA: magic multiplier (Granlund-Montgomery round-up method)
+  uint32_t dsh1;      //        min(l, 1)
+  uint32_t dsh2;      //        max(l - 1, 0), l = ceil(log2 delta)
+  uint32_t logm;      // ceil(log2 m): ballot rounds (Alg. 2 line 4) and search steps
+  uint32_t id_bytes;  // IDS: 1 or 4
+  uint32_t validate;  // IDS: flag ids >= m
+  uint32_t spl[kMaxM];
+};
+
+// id = (k >> shift) & (m - 1)
+__device__ __forceinline__ uint32_t id_lowbits(uint32_t k, const BucketParams &p) {
+  return (k >> p.shift) & p.mmask;
+}
+
+// id = min(floor(k / delta), m - 1), exact for every 32-bit k and delta >= 1:
+// q = (t + ((k - t) >> sh1)) >> sh2 with t = umulhi(k, mul).
+__device__ __forceinline__ uint32_t id_delta(uint32_t k, const BucketParams &p) {
+  uint32_t t = __umulhi(k, p.dmul);
+  uint32_t q = (t + ((k - t) >> p.dsh1)) >> p.dsh2;
+  return min(q, p.mmask);
+}
+
+// id = #{ j : s_j < k }: branchless binary search over the padded table.
+__device__ __forceinline__ uint32_t id_splitters(uint32_t k, const uint32_t *S, uint32_t logm) {
+  uint32_t pos = 0;
+#pragma unroll
+  for (int s = 7; s >= 0; --s) {
+    if ((uint32_t)s < logm) {
+      uint32_t h = 1u << s;
+      pos += (S[pos + h - 1] < k) ? h : 0u;
+    }
+  }
+  return pos;
+}
+
+template <int KIND>
+__device__ __forceinline__ uint32_t bucket_of_key(uint32_t k, const BucketParams &p,
+                                                  const uint32_t *spl_s) {
+  if constexpr (KIND == LOWBITS) return id_lowbits(k, p);
+  else if constexpr (KIND == DELTA) return id_delta(k, p);
+  else if constexpr (KIND == SPLITTERS) return id_splitters(k, spl_s, p.logm);
+  else return 0u;
+}
+
+// Precomputed id (MS_IDS), clamped so that a contract violation can never
+// index outside the tile's counters (the output is then unspecified, and
+// flagged when validation is on).
+__device__ __forceinline__ uint32_t load_id(const void *ids, uint64_t i, const BucketParams &p) {
+  uint32_t v = p.id_bytes == 1 ? (uint32_t)__ldg((const uint8_t *)ids + i)
+                               : __ldg((const uint32_t *)ids + i);
+  return min(v, p.mmask);
+}
+
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
+}
+
+// TMA 1-D bulk copy global -> shared (UBLKCP), completion counted on `bar`.
+// src, dst 16-byte aligned, bytes a multiple of 16.
+__device__ __forceinline__ void bulk_g2s(void *dst_smem, const void *src, uint32_t bytes,
+                                         uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst_smem)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t r;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
+  return r;
+}
+
+// 64-bit status words of the decoupled look-back: (flag << 32) | value.
+__device__ __forceinline__ uint64_t ld_status(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_status(uint64_t *p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, uint32_t lane) {
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    uint32_t t = __shfl_up_sync(0xFFFFFFFFu, v, d);
+    if (lane >= (uint32_t)d) v += t;
+  }
+  return v;
+}
+
+__device__ __forceinline__ uint32_t warp_sum(uint32_t v) {
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, d);
+  return v;
+}
+
+}  // namespace ms

@@ -1,0 +1,392 @@
+// ms_kernels.cuh -- the hot path: K1 pre-scan, K2 scan, K3 post-scan (sm_100a).
+//
+// PAPER.md §4 {prescan, scan, postscan}; Alg. 1;
+// Eq. (2) with subproblems = tiles of T = 256*R consecutive keys
+// (one CTA per tile, the paper's block-level granularity of Table 1
+// P:714-744, but with R keys per thread so that L = n/T stays small).
+#pragma once
+#include "ms_device.cuh"
+
+namespace ms {
+
+// ============================================================== K1 pre-scan
+// Per-tile bucket histogram -> column `tile` of H (bucket-major, H[j*L + l]).
+// Local step 1 of the skeleton, Alg. 1 lines P:819-824.
+//
+// B200 design: 128-bit coalesced loads (KPT keys per thread, all in flight
+// before any use); per-thread PRIVATE packed 8-bit counters in shared memory
+// (column tid of a [ceil(m/4)][256] word array: bank = tid % 32, so the
+// read-modify-write per key never conflicts and needs no atomics); then a
+// CTA reduction of the packed counters (two 16-bit lanes per word).
+// Counters cannot overflow: a thread counts <= KPT <= 32 keys.
+template <int KIND, int KPT>
+__global__ void __launch_bounds__(kThreads)
+k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
+           uint32_t L, uint32_t *__restrict__ H, const __grid_constant__ BucketParams p,
+           uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
+  constexpr int T = kThreads * KPT;
+  extern __shared__ __align__(16) uint32_t smem[];
+  uint32_t *spl_s = smem;              // kMaxM words (SPLITTERS)
+  uint32_t *cnt = smem + kMaxM;        // [nwords][256]
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t tile = blockIdx.x;
+  const uint64_t base = (uint64_t)tile * T;
+  const uint32_t nt = (uint32_t)umin64(T, n - base);
+  const uint32_t nwords = (p.m + 3) >> 2;
+
+  // K2's look-back status words are cleared here (K1 precedes K2 in the stream).
+  for (uint32_t i = tile * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
+  for (uint32_t i = tid; i < nwords * kThreads; i += kThreads) cnt[i] = 0;
+  if constexpr (KIND == SPLITTERS) {
+    for (uint32_t i = tid; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
+  }
+  __syncthreads();
+
+  uint32_t bad = 0;
+  auto count = [&](uint32_t id) {
+    uint32_t *c = cnt + (id >> 2) * kThreads + tid;
+    *c += 1u << ((id & 3u) * 8u);
+  };
+  if (nt == T) {
+    const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
+    uint4 v[KPT / 4];
+#pragma unroll
+    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldcs(k4 + j * kThreads + tid);  // streaming
+    if constexpr (KIND == IDS) {
+#pragma unroll
+      for (int j = 0; j < KPT / 4; ++j) {
+        uint64_t i0 = base + 4ull * (j * kThreads + tid);
+        uint32_t raw[4];
+        if (p.id_bytes == 1) {
+          uint32_t w = __ldg(reinterpret_cast<const uint32_t *>((const uint8_t *)ids + i0));
+          raw[0] = w & 255u; raw[1] = (w >> 8) & 255u; raw[2] = (w >> 16) & 255u; raw[3] = w >> 24;
+        } else {
+          uint4 w = __ldg(reinterpret_cast<const uint4 *>((const uint32_t *)ids + i0));
+          raw[0] = w.x; raw[1] = w.y; raw[2] = w.z; raw[3] = w.w;
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          bad |= raw[q] > p.mmask;
+          count(min(raw[q], p.mmask));
+        }
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < KPT / 4; ++j) {
+        count(bucket_of_key<KIND>(v[j].x, p, spl_s));
+        count(bucket_of_key<KIND>(v[j].y, p, spl_s));
+        count(bucket_of_key<KIND>(v[j].z, p, spl_s));
+        count(bucket_of_key<KIND>(v[j].w, p, spl_s));
+      }
+    }
+  } else {
+    for (uint32_t i = tid; i < nt; i += kThreads) {
+      uint32_t id;
+      if constexpr (KIND == IDS) {
+        uint32_t raw = p.id_bytes == 1 ? (uint32_t)((const uint8_t *)ids)[base + i]
+                                       : ((const uint32_t *)ids)[base + i];
+        bad |= raw > p.mmask;
+        id = min(raw, p.mmask);
+      } else {
+        id = bucket_of_key<KIND>(keys[base + i], p, spl_s);
+      }
+      count(id);
+    }
+  }
+  if constexpr (KIND == IDS) {
+    if (p.validate && __any_sync(0xFFFFFFFFu, bad) && lane == 0) atomicOr(err_flag, 1u);
+  }
+  __syncthreads();
+
+  // CTA reduction of the packed counters: warp w owns words w, w+8, ...
+  for (uint32_t q = warp; q < nwords; q += kWarps) {
+    uint32_t lo = 0, hi = 0;
+#pragma unroll
+    for (int j = 0; j < kThreads / 32; ++j) {
+      uint32_t x = cnt[q * kThreads + j * 32 + lane];
+      lo += x & 0x00FF00FFu;
+      hi += (x >> 8) & 0x00FF00FFu;
+    }
+    lo = warp_sum(lo);
+    hi = warp_sum(hi);
+    if (lane < 4) {
+      uint32_t b = 4 * q + lane;
+      uint32_t c = lane == 0 ? (lo & 0xFFFFu) : lane == 1 ? (hi & 0xFFFFu)
+                 : lane == 2 ? (lo >> 16) : (hi >> 16);
+      if (b < p.m) H[(uint64_t)b * L + tile] = c;
+    }
+  }
+}
+
+// ============================================================== K2 scan
+// G = exclusive scan of row-vectorised H (in place), Alg. 1 P:825-828:
+// G[j][l] = sum_{k<j} sum_l' h_{k,l'} + sum_{l'<l} h_{j,l'} (terms 1+2 of
+// Eq. 2).  Single pass, chained with a decoupled look-back over 64-bit
+// status words (flag << 32 | value); status is zeroed by K1 (or by the host
+// when the stage runs alone).  offsets[j] = G[j][0], offsets[m] = n.
+constexpr int kScanItems = 16;
+constexpr int kScanChunk = kThreads * kScanItems;
+constexpr uint64_t kFlagA = 1ull << 32;  // aggregate available
+constexpr uint64_t kFlagP = 2ull << 32;  // inclusive prefix available
+
+__global__ void __launch_bounds__(kThreads)
+k2_scan(uint32_t *__restrict__ data, uint64_t total, uint64_t *__restrict__ status,
+        uint32_t *__restrict__ offsets, uint32_t L, uint32_t m, uint32_t n) {
+  __shared__ uint32_t buf[kScanChunk + kScanChunk / 32];
+  __shared__ uint32_t wsum[kWarps];
+  __shared__ uint32_t prefix_s;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t chunk = blockIdx.x;
+  const uint64_t base = chunk * kScanChunk;
+  const uint32_t cnt = (uint32_t)umin64(kScanChunk, total - base);
+
+#pragma unroll
+  for (int j = 0; j < kScanItems; ++j) {
+    uint32_t i = j * kThreads + tid;
+    buf[i + (i >> 5)] = i < cnt ? data[base + i] : 0u;
+  }
+  __syncthreads();
+  uint32_t v[kScanItems];
+  uint32_t s = 0;
+#pragma unroll
+  for (int q = 0; q < kScanItems; ++q) {
+    uint32_t i = tid * kScanItems + q;
+    v[q] = buf[i + (i >> 5)];
+    s += v[q];
+  }
+  uint32_t incl = warp_incl_scan(s, lane);
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  uint32_t wpre = 0, agg = 0;
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) {
+    uint32_t x = wsum[w];
+    wpre += (w < (int)warp) ? x : 0u;
+    agg += x;
+  }
+  uint32_t texcl = wpre + incl - s;
+
+  if (chunk == 0) {
+    if (tid == 0) {
+      st_status(status, kFlagP | agg);
+      prefix_s = 0;
+    }
+  } else {
+    if (tid == 0) st_status(status + chunk, kFlagA | agg);
+    if (warp == 0) {
+      uint32_t excl = 0;
+      int64_t pred = (int64_t)chunk - 1;
+      while (true) {
+        int64_t idx = pred - lane;
+        uint64_t st = idx >= 0 ? ld_status(status + idx) : kFlagP;
+        while (__any_sync(0xFFFFFFFFu, (st >> 32) == 0)) {
+          if ((st >> 32) == 0) st = ld_status(status + idx);
+        }
+        uint32_t pmask = __ballot_sync(0xFFFFFFFFu, (st >> 32) == 2);
+        uint32_t val = (uint32_t)st;
+        if (pmask) {
+          uint32_t first = __ffs(pmask) - 1;
+          excl += warp_sum(lane <= first ? val : 0u);
+          break;
+        }
+        excl += warp_sum(val);
+        pred -= 32;
+      }
+      if (lane == 0) {
+        st_status(status + chunk, kFlagP | (uint32_t)(excl + agg));
+        prefix_s = excl;
+      }
+    }
+  }
+  __syncthreads();
+  uint32_t run = prefix_s + texcl;
+#pragma unroll
+  for (int q = 0; q < kScanItems; ++q) {
+    uint32_t i = tid * kScanItems + q;
+    buf[i + (i >> 5)] = run;
+    run += v[q];
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < kScanItems; ++j) {
+    uint32_t i = j * kThreads + tid;
+    if (i < cnt) {
+      uint64_t g = base + i;
+      uint32_t out = buf[i + (i >> 5)];
+      data[g] = out;
+      if (offsets != nullptr && (g % L) == 0) offsets[g / L] = out;
+    }
+  }
+  if (offsets != nullptr && chunk == 0 && tid == 0) offsets[m] = n;
+}
+
+// ============================================================== K3 post-scan
+// Recompute ids (footnote 6), stable tile-local ranks, a local
+// stable multisplit of the tile in shared memory (§4 "reordering",
+// P:689-713; §5.2.2 block-level reordering P:1262-1301) and coalesced stores
+// of each bucket run to G[j][tile] + (slot - S_t[j]).
+//
+// Tile = 8 warps x R rounds x 32 keys; warp w owns the contiguous segment
+// [w*32R, (w+1)*32R) and walks it in rounds of 32 consecutive keys, so
+// (warp, round, lane) order IS input order and ranks are stable.
+// Per round: logm ballots give each lane the mask of same-bucket lanes
+// (Alg. 3 with the exclusive-rank fix, reading #4); the highest
+// lane of each bucket group advances the warp's smem counter (Alg. 2's
+// histogram, accumulated).  Cross-warp exclusive prefixes + the tile's
+// bucket starts S_t then give each key its shared-memory slot (Eq. (2)
+// applied one level down).
+// Keys (and values) arrive by one TMA bulk copy per array (UBLKCP).
+template <int KIND, bool KV, int R>
+__global__ void __launch_bounds__(kThreads)
+k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
+            const void *__restrict__ ids, const uint32_t *__restrict__ G,
+            uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
+            uint32_t L, const __grid_constant__ BucketParams p) {
+  constexpr int T = kThreads * R;
+  constexpr int SEG = 32 * R;
+  constexpr bool NEED_ID8 = (KIND == SPLITTERS || KIND == IDS);
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  uint32_t *keys_s = reinterpret_cast<uint32_t *>(smem_raw);
+  uint32_t *vals_s = keys_s + T;
+  uint32_t *cnt_s = vals_s + (KV ? T : 0);     // [8][256] per-warp counters
+  uint32_t *gD_s = cnt_s + kWarps * kMaxM;     // [256] G[j][tile] - S_t[j]
+  uint32_t *spl_s = gD_s + kMaxM;              // [256] padded splitters
+  uint8_t *id8_s = reinterpret_cast<uint8_t *>(spl_s + kMaxM);  // [T]
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ uint32_t wsum[kWarps];
+
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t tile = blockIdx.x;
+  const uint64_t base = (uint64_t)tile * T;
+  const uint32_t nt = (uint32_t)umin64(T, n - base);
+  const bool full = (nt == T);
+  const uint32_t m = p.m;
+
+  if (full) {
+    if (tid == 0) {
+      mbar_init(&bar, 1);
+      fence_mbar_init();
+      mbar_arrive_expect_tx(&bar, (KV ? 2u : 1u) * T * 4u);
+      bulk_g2s(keys_s, keys + base, T * 4u, &bar);
+      if constexpr (KV) bulk_g2s(vals_s, vals + base, T * 4u, &bar);
+    }
+  } else {
+    for (uint32_t i = tid; i < nt; i += kThreads) {
+      keys_s[i] = keys[base + i];
+      if constexpr (KV) vals_s[i] = vals[base + i];
+    }
+  }
+  // per-bucket setup while the copy is in flight
+  uint32_t gcol = 0;
+  if (tid < m) gcol = __ldg(G + (uint64_t)tid * L + tile);
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] = 0;  // kThreads == kMaxM
+  if constexpr (KIND == SPLITTERS) {
+    if (tid < (1u << p.logm)) spl_s[tid] = p.spl[tid];
+  }
+  __syncthreads();
+  if (full) mbar_wait(&bar, 0);
+
+  // ---- phase 1: stable ranks within the warp's segment
+  const uint32_t lt = lanemask_lt();
+  uint32_t kreg[R];
+  uint32_t vreg[KV ? R : 1];
+  uint32_t pk[R];  // (rank within warp segment) << 8 | id
+  uint32_t *cnt_w = cnt_s + warp * kMaxM;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t pos = warp * SEG + r * 32 + lane;
+    const bool valid = full || pos < nt;
+    const uint32_t key = keys_s[pos];
+    uint32_t id = 0;
+    if (valid) {
+      if constexpr (KIND == IDS) id = load_id(ids, base + pos, p);
+      else id = bucket_of_key<KIND>(key, p, spl_s);
+    }
+    uint32_t peers = full ? 0xFFFFFFFFu : __ballot_sync(0xFFFFFFFFu, valid);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if ((uint32_t)k < p.logm) {
+        const uint32_t bit = (id >> k) & 1u;
+        const uint32_t b = __ballot_sync(0xFFFFFFFFu, bit);
+        peers &= bit ? b : ~b;
+      }
+    }
+    const uint32_t rank = __popc(peers & lt);
+    uint32_t before = 0;
+    if (valid) before = cnt_w[id];
+    __syncwarp();
+    if (valid && (peers >> lane) == 1u) cnt_w[id] = before + __popc(peers);
+    __syncwarp();
+    kreg[r] = key;
+    if constexpr (KV) vreg[r] = vals_s[pos];
+    pk[r] = ((before + rank) << 8) | id;
+  }
+  __syncthreads();
+
+  // ---- per-bucket cross-warp exclusive prefix, tile bucket starts S_t
+  uint32_t tot = 0;
+  if (tid < m) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) {
+      uint32_t c = cnt_s[w * kMaxM + tid];
+      cnt_s[w * kMaxM + tid] = tot;
+      tot += c;
+    }
+  }
+  const uint32_t incl = warp_incl_scan(tot, lane);
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  uint32_t wpre = 0;
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) wpre += (w < (int)warp) ? wsum[w] : 0u;
+  const uint32_t S = wpre + incl - tot;  // exclusive scan of tile histogram
+  if (tid < m) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] += S;
+    gD_s[tid] = gcol - S;
+  }
+  __syncthreads();
+
+  // ---- local multisplit of the tile into shared memory
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t pos = warp * SEG + r * 32 + lane;
+    if (full || pos < nt) {
+      const uint32_t id = pk[r] & 255u;
+      const uint32_t slot = cnt_w[id] + (pk[r] >> 8);
+      keys_s[slot] = kreg[r];
+      if constexpr (KV) vals_s[slot] = vreg[r];
+      if constexpr (NEED_ID8) id8_s[slot] = (uint8_t)id;
+    }
+  }
+  __syncthreads();
+
+  // ---- coalesced stores of the bucket runs
+  for (uint32_t i = tid; i < nt; i += kThreads) {
+    const uint32_t k = keys_s[i];
+    uint32_t id;
+    if constexpr (NEED_ID8) id = id8_s[i];
+    else id = bucket_of_key<KIND>(k, p, spl_s);
+    const uint32_t dst = gD_s[id] + i;
+    __stcs(keys_out + dst, k);
+    if constexpr (KV) __stcs(vals_out + dst, vals_s[i]);
+  }
+}
+
+// ============================================================== whatBucket() only
+template <int KIND>
+__global__ void __launch_bounds__(kThreads)
+k_bucket_ids(const uint32_t *__restrict__ keys, uint64_t n, uint32_t *__restrict__ out,
+             const __grid_constant__ BucketParams p) {
+  __shared__ uint32_t spl_s[kMaxM];
+  if constexpr (KIND == SPLITTERS) {
+    for (uint32_t i = threadIdx.x; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
+    __syncthreads();
+  }
+  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * kThreads)
+    out[i] = bucket_of_key<KIND>(keys[i], p, spl_s);
+}
+
+}  // namespace ms

@@ -1,0 +1,121 @@
+"""C ABI on CPU: libms.so loads, exports every symbol include/ms.h declares, and rejects bad
+arguments synchronously (before any CUDA call -- these tests run without a GPU)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+from paper_conf_ppopp_ashkianidmo16_b200 import _abi
+from paper_conf_ppopp_ashkianidmo16_b200.api import BucketSpec
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "ms.h")
+
+
+def _declared():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(ms_[a-z_]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol():
+    L = _abi.lib()
+    names = _declared()
+    assert len(names) >= 10
+    for name in names:
+        assert hasattr(L, name), f"libms.so does not export {name}"
+    assert set(names) == set(_abi.EXPORTS)
+
+
+def _create(spec: BucketSpec, max_n=1 << 20, kv=0, flags=0):
+    h = ctypes.c_void_p()
+    c = spec._c()
+    st = _abi.lib().ms_plan_create(ctypes.byref(h), ctypes.byref(c), max_n, kv, flags)
+    return st, h
+
+
+@pytest.mark.parametrize("spec,flags", [
+    (BucketSpec("lowbits", 0), 0),
+    (BucketSpec("lowbits", 257), 0),
+    (BucketSpec("lowbits", 3), 0),                 # reading #10: low-bit needs 2^k buckets
+    (BucketSpec("lowbits", 4, shift=31), 0),       # shift + log2 m > 32
+    (BucketSpec("delta", 8, delta=0), 0),
+    (BucketSpec("splitters", 3, splitters=[5, 4]), 0),   # not non-decreasing
+    (BucketSpec("ids", 8, id_bytes=2), 0),
+    (BucketSpec("delta", 8, delta=5), 2 | 4),      # two variants forced
+    (BucketSpec("delta", 8, delta=5), 64),         # unknown flag
+])
+def test_plan_create_rejects(spec, flags):
+    st, h = _create(spec, flags=flags)
+    assert st == _abi.MS_ERR_INVALID_ARG and not h.value
+
+
+def test_plan_create_rejects_huge_n():
+    st, _ = _create(BucketSpec("delta", 8, delta=5), max_n=1 << 32)
+    assert st == _abi.MS_ERR_INVALID_ARG
+
+
+@pytest.mark.parametrize("spec", [BucketSpec("lowbits", 1), BucketSpec("lowbits", 256, shift=24),
+                                  BucketSpec("delta", 256, delta=1 << 24),
+                                  BucketSpec("splitters", 3, splitters=[7, 7]),
+                                  BucketSpec("ids", 256, id_bytes=4)])
+def test_plan_create_accepts(spec):
+    st, h = _create(spec)
+    assert st == _abi.MS_OK and h.value
+    _abi.lib().ms_plan_destroy(h)
+
+
+def test_geometry_and_workspace():
+    L = _abi.lib()
+    st, h = _create(BucketSpec("delta", 32, delta=1 << 27), max_n=1 << 28)
+    for n in [1, 1 << 20, (1 << 25) + 1, 1 << 28]:
+        t, nt, v = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_int32()
+        assert L.ms_plan_geometry(h, n, ctypes.byref(t), ctypes.byref(nt), ctypes.byref(v)) == 0
+        assert nt.value == (n + t.value - 1) // t.value
+        assert t.value % 256 == 0 and 2048 <= t.value <= 8192
+        b = ctypes.c_size_t()
+        assert L.ms_plan_workspace_size(h, n, ctypes.byref(b)) == 0
+        assert b.value >= 32 * nt.value * 4                    # holds H (m x L u32)
+        bh = ctypes.c_size_t()
+        assert L.ms_plan_workspace_size_host(h, n, ctypes.byref(bh)) == 0 and bh.value >= b.value + 2 * 4 * n
+    assert L.ms_plan_workspace_size(h, (1 << 28) + 1, ctypes.byref(ctypes.c_size_t())) == _abi.MS_ERR_INVALID_ARG
+    L.ms_plan_destroy(h)
+
+
+def test_run_argument_errors_without_gpu():
+    """All of these must be refused before anything touches CUDA."""
+    L = _abi.lib()
+    st, h = _create(BucketSpec("delta", 8, delta=5), max_n=4096, kv=0)
+    P = ctypes.c_void_p
+    A, B, W = P(0x10000000), P(0x20000000), P(0x30000000)
+    big = 1 << 20
+    run = lambda k, v, i, ko, vo, n, off, ws, wsb: L.ms_run(h, k, v, i, ko, vo, n, off, ws, wsb, None)
+    assert run(None, None, None, B, None, 100, None, W, big) == _abi.MS_ERR_INVALID_ARG      # null keys
+    assert run(A, None, None, B, None, 5000, None, W, big) == _abi.MS_ERR_INVALID_ARG        # n > max_n
+    assert run(P(0x10000004), None, None, B, None, 100, None, W, big) == _abi.MS_ERR_ALIGNMENT
+    assert run(A, None, None, P(0x20000008), None, 100, None, W, big) == _abi.MS_ERR_ALIGNMENT
+    assert run(A, None, None, P(0x10000010), None, 100, None, W, big) == _abi.MS_ERR_ALIAS    # overlaps keys_in
+    assert run(A, A, None, B, B, 100, None, W, big) == _abi.MS_ERR_UNSUPPORTED             # values on KO plan
+    assert run(A, A, None, B, None, 100, None, W, big) == _abi.MS_ERR_INVALID_ARG           # unpaired values
+    assert run(A, None, None, B, None, 100, None, W, 16) == _abi.MS_ERR_WORKSPACE
+    assert run(A, None, None, B, None, 100, None, None, big) == _abi.MS_ERR_WORKSPACE
+    L.ms_plan_destroy(h)
+    st, h2 = _create(BucketSpec("ids", 8, id_bytes=1), max_n=4096)
+    assert L.ms_run(h2, A, None, None, B, None, 100, None, W, big, None) == _abi.MS_ERR_INVALID_ARG  # ids missing
+    L.ms_plan_destroy(h2)
+
+
+def test_status_strings():
+    for s in [0, -1, -2, -3, -4, -5, -6, -8]:
+        assert _abi.status_string(s) and _abi.status_string(s) != "unknown status"
+
+
+def test_product_path_has_no_oracle_or_fallback():
+    """The product package never imports the oracle and has no CPU fallback."""
+    pkg = os.path.join(ROOT, "paper_conf_ppopp_ashkianidmo16_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                src = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in src and "from oracle" not in src and "liboracle" not in src, f

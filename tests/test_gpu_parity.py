@@ -1,0 +1,213 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, bit for bit.
+
+Every comparison is element-wise and exact (integer work; the stable result
+is unique).  Inputs come from the seeded generators (workloads/); expected
+values only from oracle/ (or, for the bucket functors, the closed form).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from msutil import from_dev, make_case, to_dev
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+def _pkg():
+    import paper_conf_ppopp_ashkianidmo16_b200 as P
+    return P
+
+
+def _run_case(case, variant=None, want_offsets=True):
+    P = _pkg()
+    spec = P.BucketSpec(**case["spec_kw"])
+    n = len(case["keys"])
+    plan = P.Plan(spec, max(n, 1), with_values=case["vals"] is not None, variant=variant)
+    ko, vo, off = plan.run(to_dev(case["keys"]), to_dev(case["vals"]), to_dev(case["ids"]),
+                           want_offsets=want_offsets)
+    torch.cuda.synchronize()
+    return from_dev(ko), from_dev(vo), (None if off is None else from_dev(off)), plan
+
+
+def _expect(case):
+    return oracle.multisplit(case["ospec"], case["keys"], case["vals"], ids=case["ids"])
+
+
+def _assert_equal(case, got, exp, what=""):
+    ko, vo, off, _ = got
+    eko, evo, eoff = exp
+    assert np.array_equal(ko, eko), f"keys differ {what}: first at {np.flatnonzero(ko != eko)[:5]}"
+    if evo is not None:
+        assert np.array_equal(vo, evo), f"vals differ {what}: first at {np.flatnonzero(vo != evo)[:5]}"
+    if off is not None:
+        assert np.array_equal(off.astype(np.uint64), eoff), f"offsets differ {what}"
+
+
+NS = [0, 1, 31, 2047, 2048, 2049, 4095, 4097, 8191, 8193, 100003]
+MS = [1, 2, 3, 5, 8, 31, 32, 33, 64, 127, 255, 256]
+
+
+@pytest.mark.parametrize("kind", ["lowbits", "delta", "splitters", "ids"])
+@pytest.mark.parametrize("m", MS)
+def test_parity_matrix(kind, m):
+    """kind x m x n (empty, ragged, tile edges) x KO/KV, uniform keys."""
+    if kind == "lowbits" and m & (m - 1):
+        pytest.skip("low-bit buckets need a power-of-two m (reading #10)")
+    for i, n in enumerate(NS):
+        for kv in (False, True):
+            case = make_case(kind, m, n, seed=1000 * m + i, kv=kv, id_bytes=1 if i % 2 else 4)
+            _assert_equal(case, _run_case(case), _expect(case), f"{kind} m={m} n={n} kv={kv}")
+
+
+@pytest.mark.parametrize("dist", ["buckets", "binomial", "hot", "one"])
+@pytest.mark.parametrize("kind,m", [("lowbits", 2), ("delta", 8), ("splitters", 32), ("ids", 32),
+                                    ("delta", 256), ("splitters", 255)])
+def test_parity_distributions(kind, m, dist):
+    """Skewed workloads (§6.5): binomial, 75 % hot bucket, all in one bucket."""
+    for n in (4097, (1 << 20) + 7):
+        case = make_case(kind, m, n, seed=7 + m, dist=dist, kv=True)
+        _assert_equal(case, _run_case(case), _expect(case), f"{kind} m={m} {dist} n={n}")
+
+
+@pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("lowbits", 32, True)])
+def test_parity_2p25(kind, m, kv):
+    """BJ configs C2 / C3 size (n = 2^25), full element-wise compare."""
+    case = make_case(kind, m, 1 << 25, seed=W.SEEDS["C3"], kv=kv, vals_kind="random")
+    _assert_equal(case, _run_case(case), _expect(case), f"2^25 {kind} m={m}")
+
+
+@pytest.mark.parametrize("kv", [False, True])
+def test_parity_2p28_m256(kv):
+    """BJ config C4 (n = 2^28, m = 256, DELTA = 2^24), full element-wise compare."""
+    n = 1 << 28
+    keys = W.keys_np(n, W.SEEDS["C4"])
+    vals = W.values_np(n, W.SEEDS["C4"], "random") if kv else None
+    case = dict(spec_kw=dict(kind="delta", m=256, delta=1 << 24), ospec=oracle.Spec("delta", 256, delta=1 << 24),
+                keys=keys, vals=vals, ids=None)
+    _assert_equal(case, _run_case(case), _expect(case), "2^28 m=256")
+
+
+def test_intermediates_H_G_offsets():
+    """K1 / K2 intermediates vs the CPU Eq. (2) evaluation with the GPU's tile size T."""
+    P = _pkg()
+    for kind, m, n in [("delta", 8, 100003), ("splitters", 32, (1 << 20) + 7), ("lowbits", 256, 3 * 8192 + 5),
+                       ("ids", 17, 50000)]:
+        case = make_case(kind, m, n, seed=m + n, kv=False)
+        plan = P.Plan(P.BucketSpec(**case["spec_kw"]), n)
+        T, L, _ = plan.geometry(n)
+        kd, idd = to_dev(case["keys"]), to_dev(case["ids"])
+        H = plan.prescan(kd, idd)
+        Hh = from_dev(H).reshape(m, L).copy()
+        ids = oracle.bucket_ids(case["ospec"], case["keys"], ids=case["ids"])
+        eH, eG = oracle.tile_matrices(ids, m, T)
+        assert np.array_equal(Hh, eH), f"H differs {kind} m={m}"
+        off = torch.empty(m + 1, dtype=torch.int32, device="cuda")
+        plan.scan(H, n, off)
+        assert np.array_equal(from_dev(H).reshape(m, L), eG), f"G differs {kind} m={m}"
+        _, _, eoff = oracle.multisplit(case["ospec"], case["keys"], ids=case["ids"])
+        assert np.array_equal(from_dev(off).astype(np.uint64), eoff)
+        ko, _ = plan.postscan(kd, H, ids=idd)
+        assert np.array_equal(from_dev(ko), oracle.multisplit(case["ospec"], case["keys"], ids=case["ids"])[0])
+
+
+def test_scan_many_chunks():
+    """K2 look-back across many chunks (m*L >> 4096) against numpy's exclusive cumsum of H."""
+    P = _pkg()
+    n = 1 << 24
+    plan = P.Plan(P.BucketSpec.delta_range(256, 1 << 24), n)
+    T, L, _ = plan.geometry(n)
+    rng = np.random.default_rng(0)
+    H = rng.integers(0, 60, size=256 * L).astype(np.uint32)
+    exp = np.concatenate([[0], np.cumsum(H.astype(np.uint64))[:-1]]).astype(np.uint32)
+    d = to_dev(H)
+    plan.scan(d, n)
+    assert np.array_equal(from_dev(d), exp)
+
+
+def test_torch_stable_sort_cross_check():
+    """Independent GPU cross-check: torch.sort(ids, stable=True) + gather (the RBS analogue, §3.4)."""
+    P = _pkg()
+    n, m, delta = (1 << 22) + 3, 8, 400000000
+    keys = W.keys_torch(n, 5, "cuda")
+    vals = W.values_torch(n, 5, "cuda", "random")
+    ko, vo, off = P.multisplit(keys, vals, P.BucketSpec.delta_range(m, delta))
+    k64 = keys.to(torch.int64) & 0xFFFFFFFF
+    ids = torch.clamp(k64 // delta, max=m - 1)
+    _, idx = torch.sort(ids, stable=True)
+    assert torch.equal(ko, keys[idx]) and torch.equal(vo, vals[idx])
+
+
+@pytest.mark.parametrize("delta", [1, 3, 7, 400000000, 1 << 24, 0xFFFFFFFF, 0x80000001, 65535])
+def test_delta_functor_exhaustive(delta):
+    """Device DELTA functor == min(k // delta, m-1) for EVERY 32-bit key (exact magic division)."""
+    P = _pkg()
+    m = 256
+    plan = P.Plan(P.BucketSpec.delta_range(m, delta), 1 << 30)
+    chunk = 1 << 30
+    for c in range(4):
+        k64 = torch.arange(c * chunk, (c + 1) * chunk, dtype=torch.int64, device="cuda")
+        keys = (k64 - ((k64 >> 31) << 32)).to(torch.int32)
+        got = plan.bucket_ids(keys)
+        exp = torch.clamp(k64 // delta, max=m - 1).to(torch.int32)
+        assert torch.equal(got, exp), f"delta={delta} chunk {c}"
+        del k64, keys, got, exp
+
+
+def test_splitter_functor_dense():
+    """Device splitter search == #{j: s_j < k} on keys at and around every splitter (incl. duplicates)."""
+    P = _pkg()
+    for m in (2, 3, 32, 200, 256):
+        spl = sorted(W.gen_splitters(m, m).tolist())
+        if m > 3:
+            spl[1] = spl[2]
+        keys = sorted({0, 1, 0xFFFFFFFF} | {s + d for s in spl for d in (-1, 0, 1) if 0 <= s + d <= 0xFFFFFFFF})
+        kn = np.array(keys, dtype=np.uint32)
+        plan = P.Plan(P.BucketSpec.from_splitters(spl), len(kn))
+        got = from_dev(plan.bucket_ids(to_dev(kn)))
+        exp = np.searchsorted(np.array(spl, dtype=np.uint64), kn.astype(np.uint64), side="left")
+        assert np.array_equal(got, exp.astype(np.uint32))
+
+
+def test_validate_flags_out_of_range_ids():
+    P = _pkg()
+    n, m = 10000, 16
+    ids = W.bucket_draw_np(n, 1, "buckets", m)
+    keys = W.keys_np(n, 1)
+    plan = P.Plan(P.BucketSpec.precomputed(m, 1), n, validate=True)
+    plan.run(to_dev(keys), ids=to_dev(ids))
+    assert plan.check() == 0
+    bad = ids.copy()
+    bad[777] = 200
+    plan.run(to_dev(keys), ids=to_dev(bad))
+    assert plan.check() == -8
+    plan.run(to_dev(keys), ids=to_dev(ids))
+    assert plan.check() == 0
+
+
+def test_run_host_matches_oracle():
+    """ms_run_host (host buffers, copies inside the call) == oracle."""
+    P = _pkg()
+    case = make_case("splitters", 32, (1 << 20) + 9, seed=3, kv=True, vals_kind="random")
+    plan = P.Plan(P.BucketSpec(**case["spec_kw"]), len(case["keys"]), with_values=True)
+    kh = torch.from_numpy(case["keys"].view(np.int32).copy()).pin_memory()
+    vh = torch.from_numpy(case["vals"].view(np.int32).copy()).pin_memory()
+    ko, vo, off = plan.run_host(kh, vh)
+    eko, evo, eoff = _expect(case)
+    assert np.array_equal(ko.numpy().view(np.uint32), eko)
+    assert np.array_equal(vo.numpy().view(np.uint32), evo)
+    assert np.array_equal(off.numpy().view(np.uint32).astype(np.uint64), eoff)
+
+
+def test_repeated_runs_same_workspace():
+    """Look-back status is re-zeroed each run: repeated runs on one workspace stay exact."""
+    P = _pkg()
+    case = make_case("delta", 256, (1 << 21) + 1, seed=9, kv=True)
+    plan = P.Plan(P.BucketSpec(**case["spec_kw"]), len(case["keys"]), with_values=True)
+    kd, vd = to_dev(case["keys"]), to_dev(case["vals"])
+    exp = _expect(case)
+    for _ in range(3):
+        ko, vo, off = plan.run(kd, vd)
+        assert np.array_equal(from_dev(ko), exp[0]) and np.array_equal(from_dev(vo), exp[1])

@@ -23,6 +23,7 @@ over equal-width buckets; §6.5 P:2147-2170 binomial B(m-1, 1/2) and
 * ``buckets``   b uniform over [0, m), then key uniform in range(b).
 * ``binomial``  b = popcount of (m-1) random bits (exactly B(m-1, 1/2)).
 * ``hot``       with prob 3/4 b = m // 2, else b uniform; key uniform in range(b).
+* ``one``       every key in bucket m // 2 (degenerate case: one non-empty bucket).
 """
 from __future__ import annotations
 
@@ -87,6 +88,8 @@ def draw_buckets_np(dist: str, m: int, seed: int, start: int, n: int) -> np.ndar
         hot = (r & np.uint64(3)) != 0
         u = ((((r >> np.uint64(32)) * np.uint64(m)) >> np.uint64(32))).astype(np.uint32)
         return np.where(hot, np.uint32(m // 2), u).astype(np.uint32)
+    if dist == "one":
+        return np.full(n, m // 2, dtype=np.uint32)
     raise ValueError(dist)
 
 
@@ -148,6 +151,8 @@ def draw_buckets_torch(dist, m, seed, start, n, device):
         hot = torch.bitwise_and(r, 3) != 0
         u = (_srl(r, 32) * m) >> 32
         return torch.where(hot, torch.full_like(u, m // 2), u)
+    if dist == "one":
+        return torch.full((n,), m // 2, dtype=torch.int64, device=device)
     raise ValueError(dist)
 
 
