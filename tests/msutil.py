@@ -22,7 +22,7 @@ def make_case(kind: str, m: int, n: int, seed: int, dist: str = "uniform", kv: b
         if m == 1:
             spec_kw["shift"] = shift = 0
     elif kind == "delta":
-        delta = max(1, (1 << 32) // m) if seed % 2 == 0 else 400000000
+        delta = min(0xFFFFFFFF, max(1, (1 << 32) // m)) if seed % 2 == 0 else 400000000
         spec_kw["delta"] = delta
         ranges = W.ranges_delta(m, delta)
     elif kind == "splitters":
