@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libms.so")
 SOURCES = ["ms_api.cu"]
-DEPS = SOURCES + ["ms_kernels.cuh", "ms_device.cuh", "ms_onepass.cuh"]
+DEPS = SOURCES + ["ms_kernels.cuh", "ms_device.cuh", "ms_k3_blocked.cuh", "ms_onepass.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
          "-Xcompiler", "-fPIC", "-shared", "-cudart", "static", "--expt-relaxed-constexpr"]

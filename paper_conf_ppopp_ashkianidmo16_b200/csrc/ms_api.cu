@@ -8,12 +8,14 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
 
 #include "../../include/ms.h"
 #include "ms_kernels.cuh"
+#include "ms_k3_blocked.cuh"
 
 using namespace ms;
 
@@ -23,6 +25,8 @@ struct ms_plan_s {
   int kv;
   uint32_t flags;
   BucketParams bp;
+  int kkind;  // kernel-level Kind (ms_device.cuh)
+  int reverse = 0;  // K3 walks tiles last-to-first (L2 reuse of K1's tail)
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
   int tracing = 0;
@@ -55,21 +59,18 @@ uint32_t ceil_log2(uint32_t m) {
   return l;
 }
 
-// Granlund & Montgomery round-up division by an invariant (1 <= d < 2^32):
-// q = (t + ((k - t) >> sh1)) >> sh2,  t = umulhi(k, mul).
-void delta_magic(uint32_t d, uint32_t *mul, uint32_t *sh1, uint32_t *sh2) {
-  uint32_t l = ceil_log2(d);
-  uint64_t num = ((1ull << 32) * ((1ull << l) - d)) / d + 1;  // < 2^32 for d >= 1
-  *mul = (uint32_t)num;
-  *sh1 = l < 1 ? l : 1;
-  *sh2 = l > 0 ? l - 1 : 0;
-}
+// Division by an invariant 32-bit delta that is not a power of two (so
+// delta >= 3): c = ceil(2^64 / delta) = floor((2^64 - 1) / delta) + 1, and
+// floor(k / delta) = floor(k * c / 2^64) for every 32-bit k (Lemire, Kaser &
+// Kurz: exact when the magic has >= 32 + log2(delta) fractional bits).
+uint64_t delta_magic(uint32_t d) { return ~0ull / d + 1; }
 
 // Rounds per warp R (tile T = 256 R): 16 for m <= 32, 32 above (runs of T/m
 // keys stay >= 32 keys = 128 B); halved while the grid would not fill two
 // waves of 148 SMs (small n is launch/latency bound, not HBM bound).
 int rounds_for(uint32_t m, uint64_t n) {
-  int R = m <= 32 ? 16 : 32;
+  if (m <= 32) return 16;  // K3b (blocked ranks) uses T = 4096 for every n
+  int R = 16;
   while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
   return R;
 }
@@ -111,7 +112,7 @@ void set_smem(K kernel, size_t bytes) {
   if (bytes > 48 * 1024) cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
 }
 
-size_t k1_smem(uint32_t m) { return (kMaxM + ((m + 3) / 4) * kThreads) * 4; }
+size_t k1_smem(uint32_t m) { return kMaxM * 4 + (size_t)m * kThreads; }
 
 size_t k3_smem(int R, bool kv, bool id8) {
   size_t T = 256u * R;
@@ -144,7 +145,7 @@ template <int KIND, bool KV>
 cudaError_t launch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                       const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                       uint32_t *vo, uint32_t n, cudaStream_t s) {
-  constexpr bool id8 = (KIND == SPLITTERS || KIND == IDS);
+  constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC);
 #define MS_K3(R)                                                                             \
   {                                                                                          \
     auto k = k3_postscan<KIND, KV, R>;                                                       \
@@ -164,11 +165,61 @@ cudaError_t launch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *key
 cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const void *ids,
                         uint32_t n, uint32_t *H, uint64_t *zp, uint32_t zw, uint32_t *flag,
                         cudaStream_t s) {
-  switch (p->spec.kind) {
-    case MS_LOWBITS: return launch_k1<LOWBITS>(p, g, keys, ids, n, H, zp, zw, flag, s);
-    case MS_DELTA: return launch_k1<DELTA>(p, g, keys, ids, n, H, zp, zw, flag, s);
-    case MS_SPLITTERS: return launch_k1<SPLITTERS>(p, g, keys, ids, n, H, zp, zw, flag, s);
+  switch (p->kkind) {
+    case LOWBITS: return launch_k1<LOWBITS>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case SHIFTC: return launch_k1<SHIFTC>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case DELTA: return launch_k1<DELTA>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case SPLITTERS: return launch_k1<SPLITTERS>(p, g, keys, ids, n, H, zp, zw, flag, s);
     default: return launch_k1<IDS>(p, g, keys, ids, n, H, zp, zw, flag, s);
+  }
+}
+
+// Persistent grid: SM count x resident CTAs per SM (cached per kernel).
+template <typename K>
+unsigned persistent_grid(K kernel, size_t smem, uint64_t tiles) {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kThreads, smem);
+  if (per_sm <= 0) per_sm = 1;
+  return (unsigned)std::min<uint64_t>(tiles, (uint64_t)sms * per_sm);
+}
+
+template <int KIND, bool KV, int LOGMP>
+cudaError_t launch_k3b_l(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const uint32_t *vals,
+                         const void *ids, const uint32_t *G, uint32_t *ko, uint32_t *vo, uint32_t n,
+                         cudaStream_t s) {
+  if (KIND == IDS && p->spec.id_bytes == 1) {
+    auto k = k3p_postscan<KIND, KV, LOGMP, true>;
+    const size_t smem = K3pLayout<LOGMP, KV, true>::BYTES;
+    set_smem(k, smem);
+    k<<<persistent_grid(k, smem, g.L), kThreads, smem, s>>>(keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->bp,
+                                                           p->reverse);
+  } else {
+    auto k = k3p_postscan<KIND, KV, LOGMP, false>;
+    const size_t smem = K3pLayout<LOGMP, KV, false>::BYTES;
+    set_smem(k, smem);
+    k<<<persistent_grid(k, smem, g.L), kThreads, smem, s>>>(keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->bp,
+                                                           p->reverse);
+  }
+  return cudaGetLastError();
+}
+
+template <int KIND, bool KV>
+cudaError_t launch_k3b(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const uint32_t *vals,
+                       const void *ids, const uint32_t *G, uint32_t *ko, uint32_t *vo, uint32_t n,
+                       cudaStream_t s) {
+  switch (std::max<uint32_t>(1, ceil_log2(p->spec.m))) {
+    case 1: return launch_k3b_l<KIND, KV, 1>(p, g, keys, vals, ids, G, ko, vo, n, s);
+    case 2: return launch_k3b_l<KIND, KV, 2>(p, g, keys, vals, ids, G, ko, vo, n, s);
+    case 3: return launch_k3b_l<KIND, KV, 3>(p, g, keys, vals, ids, G, ko, vo, n, s);
+    case 4: return launch_k3b_l<KIND, KV, 4>(p, g, keys, vals, ids, G, ko, vo, n, s);
+    default: return launch_k3b_l<KIND, KV, 5>(p, g, keys, vals, ids, G, ko, vo, n, s);
   }
 }
 
@@ -176,13 +227,27 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                         uint32_t *vo, uint32_t n, cudaStream_t s) {
   const bool kv = vals != nullptr;
+  if (p->spec.m <= 32) {
+#define MS_K3B(KIND)                                                        \
+  return kv ? launch_k3b<KIND, true>(p, g, keys, vals, ids, G, ko, vo, n, s) \
+            : launch_k3b<KIND, false>(p, g, keys, vals, ids, G, ko, vo, n, s);
+    switch (p->kkind) {
+      case LOWBITS: MS_K3B(LOWBITS)
+      case SHIFTC: MS_K3B(SHIFTC)
+      case DELTA: MS_K3B(DELTA)
+      case SPLITTERS: MS_K3B(SPLITTERS)
+      default: MS_K3B(IDS)
+    }
+#undef MS_K3B
+  }
 #define MS_K3K(KIND)                                                     \
   return kv ? launch_k3<KIND, true>(p, g, keys, vals, ids, G, ko, vo, n, s) \
             : launch_k3<KIND, false>(p, g, keys, vals, ids, G, ko, vo, n, s);
-  switch (p->spec.kind) {
-    case MS_LOWBITS: MS_K3K(LOWBITS)
-    case MS_DELTA: MS_K3K(DELTA)
-    case MS_SPLITTERS: MS_K3K(SPLITTERS)
+  switch (p->kkind) {
+    case LOWBITS: MS_K3K(LOWBITS)
+    case SHIFTC: MS_K3K(SHIFTC)
+    case DELTA: MS_K3K(DELTA)
+    case SPLITTERS: MS_K3K(SPLITTERS)
     default: MS_K3K(IDS)
   }
 #undef MS_K3K
@@ -234,6 +299,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (flags & ~(MS_VALIDATE | MS_VARIANT_3K | MS_VARIANT_1P)) return MS_ERR_INVALID_ARG;
   BucketParams bp;
   memset(&bp, 0, sizeof(bp));
+  int kkind = spec->kind;
   bp.m = m;
   bp.mmask = m - 1;
   bp.logm = ceil_log2(m);
@@ -246,7 +312,15 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
       break;
     case MS_DELTA:
       if (spec->delta < 1) return MS_ERR_INVALID_ARG;
-      delta_magic(spec->delta, &bp.dmul, &bp.dsh1, &bp.dsh2);
+      if ((spec->delta & (spec->delta - 1)) == 0) {  // power of two (incl. 1): a shift
+        kkind = SHIFTC;
+        bp.shift = ceil_log2(spec->delta);
+      } else {
+        kkind = DELTA;
+        const uint64_t c = delta_magic(spec->delta);
+        bp.magic_lo = (uint32_t)c;
+        bp.magic_hi = (uint32_t)(c >> 32);
+      }
       break;
     case MS_SPLITTERS: {
       if (m > 1 && !spec->splitters) return MS_ERR_INVALID_ARG;
@@ -271,7 +345,10 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->kv = with_values ? 1 : 0;
   p->flags = flags;
   p->bp = bp;
+  p->kkind = kkind;
   p->last_launches = 0;
+  // ablation override: MS_K3_REVERSE=1 makes K3 walk tiles last-to-first
+  if (const char *e = getenv("MS_K3_REVERSE")) p->reverse = atoi(e) ? 1 : 0;
   *plan = p;
   return MS_OK;
 }
@@ -483,9 +560,10 @@ ms_status ms_bucket_ids(ms_plan_t p, const uint32_t *keys_in, uint64_t n, uint32
   if (n == 0) return MS_OK;
   cudaStream_t s = (cudaStream_t)stream;
   unsigned grid = (unsigned)std::min<uint64_t>((n + kThreads - 1) / kThreads, 148ull * 16);
-  switch (p->spec.kind) {
-    case MS_LOWBITS: k_bucket_ids<LOWBITS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
-    case MS_DELTA: k_bucket_ids<DELTA><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+  switch (p->kkind) {
+    case LOWBITS: k_bucket_ids<LOWBITS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+    case SHIFTC: k_bucket_ids<SHIFTC><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+    case DELTA: k_bucket_ids<DELTA><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
     default: k_bucket_ids<SPLITTERS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
   }
   return cudaGetLastError() == cudaSuccess ? MS_OK : MS_ERR_CUDA;

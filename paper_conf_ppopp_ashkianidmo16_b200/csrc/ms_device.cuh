@@ -1,31 +1,32 @@
 // ms_device.cuh -- device primitives of the B200 multisplit (sm_100a).
 //
-// Bucket functors (whatBucket()), warp vote
-// helpers (the ballot/popc machinery of Alg. 2/3, §5.1) and the
-// TMA bulk-copy + mbarrier wrappers used to stage tiles in shared memory.
+// Bucket functors (whatBucket()), warp
+// helpers and the TMA bulk-copy + mbarrier wrappers used to stage tiles in
+// shared memory.
 #pragma once
 #include <cstdint>
 
 namespace ms {
 
-enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3 };
+// Kernel-level bucket-function kinds.  The public kinds (ms.h) map onto
+// these; MS_DELTA becomes SHIFTC when delta is a power of two (incl. 1).
+enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3, SHIFTC = 4 };
 
 constexpr int kThreads = 256;  // CTA = 8 warps (the paper's NW = 8)
 constexpr int kWarps = kThreads / 32;
 constexpr int kMaxM = 256;
 
-// Bucket-function constants, passed by value as a kernel parameter (lives in
-// the constant bank; no device allocation).  spl[] holds the splitters padded
-// to Q = 2^logm entries with 0xFFFFFFFF (never "< key"), so the branchless
+// Bucket-function constants, passed by value as a kernel parameter (constant
+// bank; no device allocation).  spl[] holds the splitters padded to
+// Q = 2^logm entries with 0xFFFFFFFF (never "< key"), so the branchless
 // search below always runs exactly logm steps.
 struct BucketParams {
   uint32_t m;         // number of buckets (1..256)
   uint32_t mmask;     // m - 1
-  uint32_t shift;     // LOWBITS bit offset
-  uint32_t dmul;      // DELTA: magic multiplier (Granlund-Montgomery round-up method)
-  uint32_t dsh1;      //        min(l, 1)
-  uint32_t dsh2;      //        max(l - 1, 0), l = ceil(log2 delta)
-  uint32_t logm;      // ceil(log2 m): ballot rounds (Alg. 2 line 4) and search steps
+  uint32_t shift;     // LOWBITS bit offset; SHIFTC: log2(delta)
+  uint32_t magic_lo;  // DELTA: c = ceil(2^64 / delta) (Lemire-Kaser-Kurz), low word
+  uint32_t magic_hi;  //        high word
+  uint32_t logm;      // ceil(log2 m): splitter search steps
   uint32_t id_bytes;  // IDS: 1 or 4
   uint32_t validate;  // IDS: flag ids >= m
   uint32_t spl[kMaxM];
@@ -36,19 +37,26 @@ __device__ __forceinline__ uint32_t id_lowbits(uint32_t k, const BucketParams &p
   return (k >> p.shift) & p.mmask;
 }
 
-// id = min(floor(k / delta), m - 1), exact for every 32-bit k and delta >= 1:
-// q = (t + ((k - t) >> sh1)) >> sh2 with t = umulhi(k, mul).
+// id = min(k >> log2(delta), m - 1): delta a power of two
+__device__ __forceinline__ uint32_t id_shiftc(uint32_t k, const BucketParams &p) {
+  return min(k >> p.shift, p.mmask);
+}
+
+// id = min(floor(k / delta), m - 1) for 1 < delta < 2^32, not a power of two:
+// floor(k * c / 2^64) with c = ceil(2^64 / delta) is exact for every 32-bit k
+// (F = 64 >= N + log2(delta) = 32 + 32).  Two 32x32->64 multiply-adds.
 __device__ __forceinline__ uint32_t id_delta(uint32_t k, const BucketParams &p) {
-  uint32_t t = __umulhi(k, p.dmul);
-  uint32_t q = (t + ((k - t) >> p.dsh1)) >> p.dsh2;
-  return min(q, p.mmask);
+  const uint64_t lo = (uint64_t)p.magic_lo * k;
+  const uint64_t hi = (uint64_t)p.magic_hi * k + (lo >> 32);
+  return min((uint32_t)(hi >> 32), p.mmask);
 }
 
 // id = #{ j : s_j < k }: branchless binary search over the padded table.
+template <int LOGM_MAX = 8>
 __device__ __forceinline__ uint32_t id_splitters(uint32_t k, const uint32_t *S, uint32_t logm) {
   uint32_t pos = 0;
 #pragma unroll
-  for (int s = 7; s >= 0; --s) {
+  for (int s = LOGM_MAX - 1; s >= 0; --s) {
     if ((uint32_t)s < logm) {
       uint32_t h = 1u << s;
       pos += (S[pos + h - 1] < k) ? h : 0u;
@@ -61,6 +69,7 @@ template <int KIND>
 __device__ __forceinline__ uint32_t bucket_of_key(uint32_t k, const BucketParams &p,
                                                   const uint32_t *spl_s) {
   if constexpr (KIND == LOWBITS) return id_lowbits(k, p);
+  else if constexpr (KIND == SHIFTC) return id_shiftc(k, p);
   else if constexpr (KIND == DELTA) return id_delta(k, p);
   else if constexpr (KIND == SPLITTERS) return id_splitters(k, spl_s, p.logm);
   else return 0u;
@@ -88,6 +97,7 @@ __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
 
+// order generic-proxy shared-memory writes before later async-proxy (TMA) reads
 __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -122,11 +132,30 @@ __device__ __forceinline__ void bulk_g2s(void *dst_smem, const void *src, uint32
       : "memory");
 }
 
+// TMA 1-D bulk copy shared -> global (bulk-group completion).  dst, src
+// 16-byte aligned, bytes a multiple of 16.
+__device__ __forceinline__ void bulk_s2g(void *dst, const void *src_smem, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+               "r"(smem_u32(src_smem)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+// wait until the committed bulk stores have finished READING shared memory
+__device__ __forceinline__ void bulk_wait_read0() {
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t r;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t lanemask_gt() {
+  uint32_t r;
+  asm("mov.u32 %0, %%lanemask_gt;" : "=r"(r));
   return r;
 }
 
@@ -149,10 +178,6 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, uint32_t lane) {
   return v;
 }
 
-__device__ __forceinline__ uint32_t warp_sum(uint32_t v) {
-#pragma unroll
-  for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, d);
-  return v;
-}
+__device__ __forceinline__ uint32_t warp_sum(uint32_t v) { return __reduce_add_sync(0xFFFFFFFFu, v); }
 
 }  // namespace ms

@@ -1,0 +1,358 @@
+// ms_k3_blocked.cuh -- K3 post-scan for m <= 32: persistent, blocked ranks, TMA bulk stores (sm_100a).
+//
+// Same contract as k3_postscan (ms_kernels.cuh): recompute ids (footnote 6,
+// P:857-859), stable local offsets (term 3 of Eq. (2)), a local
+// stable multisplit of the tile in shared memory (§4 reordering, P:689-713;
+// block-level reordering §5.2.2), then bucket runs written to
+// G[j][tile] + (slot - S_t[j]).
+//
+// B200 design: no warp votes at all.  The paper's local
+// offsets come from an explicit H-bar scan (§4 "explicit" local offsets,
+// P:650-666) done hierarchically:
+//  * thread t owns the contiguous block beta(t) of 16 keys and counts them
+//    sequentially into a private column of u16 counters c[j][beta] in shared
+//    memory -- the count it reads before incrementing IS the key's stable
+//    rank inside the block; beta(t) = 2*lane + (warp & 1) + 64*(warp >> 1)
+//    puts the 32 lanes of a warp in 32 different banks whatever their ids;
+//  * one CTA-wide exclusive scan over the row-vectorised counter matrix
+//    (bucket-major, blocks in input order -- the same "row-vectorised" scan
+//    as the global one, Alg. 1) turns every counter into the
+//    key's slot in the locally multisplit tile;
+//  * bucket j's run is placed at a slot P_j congruent to its global start
+//    G_j modulo 4 keys (<= 3 padding slots per bucket), so the run body is
+//    one TMA bulk store (cp.async.bulk, UBLKCP) shared -> global; only the
+//    <= 3 + 3 unaligned head/tail keys use plain stores.
+// Persistent CTAs walk tiles with a stride of gridDim.x; each thread
+// prefetches its own next blocks with cp.async (LDGSTS) into a chunk-major
+// staging ring, so loads for the next STAGES tiles are in flight while the
+// current tile is ranked and stored, and no barrier guards the staging data.
+namespace ms {
+
+template <int LOGMP, bool KV, bool IDS8>
+struct K3pLayout {
+  static constexpr int MP = 1 << LOGMP;        // bucket rows (m rounded up to a power of 2, >= 2)
+  static constexpr int K = 16;                 // keys per thread
+  static constexpr int T = kThreads * K;       // 4096 keys per tile
+  static constexpr int STAGES = KV ? 1 : 2;    // tiles prefetched ahead
+  static constexpr int CW = MP * 128;          // counter words (MP x 256 u16)
+  static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // key slots incl. alignment padding
+  static constexpr int WPT = MP / 2;           // counter words per thread in the scan
+  static constexpr int MW = 3 * MP + 8;        // per-tile metadata words: rowS[MP+4] P[MP] G[MP]
+  // word offsets
+  static constexpr int O_CNT = 0;
+  static constexpr int O_KEYS = O_CNT + CW;
+  static constexpr int O_VALS = O_KEYS + KSR;
+  static constexpr int O_STK = O_VALS + (KV ? KSR : 0);           // [STAGES][T] keys
+  static constexpr int O_STV = O_STK + STAGES * T;                // [STAGES][T] vals
+  static constexpr int O_STI = O_STV + (KV ? STAGES * T : 0);     // [STAGES][T/4] u8 ids
+  static constexpr int O_META = O_STI + (IDS8 ? STAGES * T / 4 : 0);  // [2][MW] (tile parity)
+  static constexpr int O_WS = O_META + 2 * MW;
+  static constexpr int O_SPL = O_WS + 12;
+  static constexpr int WORDS = O_SPL + kMaxM;
+  static constexpr size_t BYTES = (size_t)WORDS * 4;
+};
+
+__device__ __forceinline__ void cp_async16(void *smem_dst, const void *src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(smem_dst)), "l"(src),
+               "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async16_full(void *smem_dst, const void *src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem_dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
+// Stage this thread's chunks of tile `tile` (keys: 4 x 16 B; vals likewise;
+// u8 ids: 1 x 16 B) into stage slot `st`, chunk-major ([c][tid]) so the
+// later 128-bit reads are conflict-free.  Bytes past n are zero-filled.
+template <bool KV, bool IDS8, int T>
+__device__ __forceinline__ void k3p_prefetch(uint32_t *stk, uint32_t *stv, uint32_t *sti, int st,
+                                             const uint32_t *keys, const uint32_t *vals, const void *ids,
+                                             uint64_t tile, uint32_t n, uint32_t beta) {
+  const uint32_t tid = threadIdx.x;
+  const uint64_t b0 = tile * T + beta * 16ull;
+  uint32_t *dk = stk + st * T + tid * 4;
+  uint32_t *dv = stv + st * T + tid * 4;
+  if (tile * T + T <= n) {
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      cp_async16_full(dk + c * kThreads * 4, keys + b0 + 4 * c);
+      if constexpr (KV) cp_async16_full(dv + c * kThreads * 4, vals + b0 + 4 * c);
+    }
+    if constexpr (IDS8) cp_async16_full(sti + st * (T / 4) + tid * 4, (const uint8_t *)ids + b0);
+  } else {
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const uint64_t e = b0 + 4 * c;
+      const uint32_t bytes = e >= n ? 0u : (uint32_t)(umin64(4, n - e) * 4);
+      const uint64_t src = bytes ? e : 0;
+      cp_async16(dk + c * kThreads * 4, keys + src, bytes);
+      if constexpr (KV) cp_async16(dv + c * kThreads * 4, vals + src, bytes);
+    }
+    if constexpr (IDS8) {
+      const uint32_t bytes = b0 >= n ? 0u : (uint32_t)umin64(16, n - b0);
+      cp_async16(sti + st * (T / 4) + tid * 4, (const uint8_t *)ids + (bytes ? b0 : 0), bytes);
+    }
+  }
+}
+
+// One tile, already staged.  FULL: all 4096 keys valid (no per-key predicates).
+template <int KIND, bool KV, int LOGMP, bool IDS8, bool FULL>
+__device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *sm_v, const uint32_t *sm_i,
+                                         const void *__restrict__ ids, uint32_t *__restrict__ keys_out,
+                                         uint32_t *__restrict__ vals_out, uint64_t base, uint32_t nt,
+                                         const BucketParams &p, uint32_t *sm, uint32_t beta, uint32_t *meta) {
+  using Ly = K3pLayout<LOGMP, KV, IDS8>;
+  constexpr int MP = Ly::MP, K = Ly::K;
+  // ids are recomputed from the key where that is cheaper than keeping them
+  constexpr bool KEEP_ID = (KIND == SPLITTERS) || (KIND == IDS && !IDS8);
+  uint32_t *cnt32 = sm + Ly::O_CNT;
+  uint32_t *keys_s = sm + Ly::O_KEYS;
+  uint32_t *vals_s = sm + Ly::O_VALS;
+  uint32_t *rowS = meta;            // [MP+4]
+  uint32_t *Pj = meta + MP + 4;     // [MP]
+  uint32_t *Gj = Pj + MP;           // [MP]
+  uint32_t *wsum = sm + Ly::O_WS;
+  const uint32_t *spl_s = sm + Ly::O_SPL;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t m = p.m;
+  const uint32_t b0 = beta * K;
+  // this thread's counter column: byte address of c[0][beta]; c[j][beta] is j*512 bytes further
+  uint8_t *cb = reinterpret_cast<uint8_t *>(cnt32) + 2 * beta;
+
+  // ---- own staged chunks -> registers
+  uint32_t k[K];
+  uint32_t v[KV ? K : 1];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint4 x = *reinterpret_cast<const uint4 *>(sm_k + (c * kThreads + tid) * 4);
+    k[4 * c] = x.x; k[4 * c + 1] = x.y; k[4 * c + 2] = x.z; k[4 * c + 3] = x.w;
+    if constexpr (KV) {
+      const uint4 y = *reinterpret_cast<const uint4 *>(sm_v + (c * kThreads + tid) * 4);
+      v[4 * c] = y.x; v[4 * c + 1] = y.y; v[4 * c + 2] = y.z; v[4 * c + 3] = y.w;
+    }
+  }
+  uint32_t idw[IDS8 ? 4 : 1];
+  if constexpr (IDS8) {
+    const uint4 x = *reinterpret_cast<const uint4 *>(sm_i + tid * 4);
+    idw[0] = x.x; idw[1] = x.y; idw[2] = x.z; idw[3] = x.w;
+  }
+  auto id_of = [&](int q) -> uint32_t {
+    if constexpr (KIND == IDS) {
+      if constexpr (IDS8) return min((idw[q >> 2] >> (8 * (q & 3))) & 255u, p.mmask);
+      else return (FULL || b0 + q < nt) ? load_id(ids, base + b0 + q, p) : 0u;
+    } else {
+      return bucket_of_key<KIND>(k[q], p, spl_s);
+    }
+  };
+
+  // ---- 1. sequential per-block counting: the rank within the block
+  uint32_t rk[2] = {0u, 0u};                 // 4-bit ranks (< 16), 8 per word
+  uint32_t idk[KEEP_ID ? 4 : 1];             // kept ids, 8 bits each
+  if constexpr (KEEP_ID) idk[0] = idk[1] = idk[2] = idk[3] = 0u;
+#pragma unroll
+  for (int q = 0; q < K; ++q) {
+    const uint32_t id = id_of(q);
+    if (FULL || b0 + q < nt) {
+      uint16_t *c = reinterpret_cast<uint16_t *>(cb + (id << 9));
+      const uint32_t r = *c;
+      *c = (uint16_t)(r + 1);
+      rk[q >> 3] += r << (4 * (q & 7));
+      if constexpr (KEEP_ID) idk[q >> 2] |= id << (8 * (q & 3));
+    }
+  }
+  __syncthreads();
+
+  // ---- 2. CTA exclusive scan of the row-vectorised counter matrix
+  // Thread t owns words [t*WPT, (t+1)*WPT) (one bucket row).  With >= 2
+  // 16-byte chunks per thread, the chunk order is rotated per lane so the
+  // 128-bit accesses of every 8-lane phase hit 8 different bank groups.
+  const uint32_t row = tid >> (8 - LOGMP);
+  constexpr int WPT = Ly::WPT;
+  constexpr int NC = WPT >= 4 ? WPT / 4 : 1;       // 16-byte chunks per thread
+  constexpr int CWD = WPT >= 4 ? 4 : WPT;          // words per chunk
+  const uint32_t rot = NC == 4 ? ((tid >> 1) & 3) : NC == 2 ? ((tid >> 2) & 1) : 0;
+  uint32_t w[NC][CWD];
+  uint32_t csum[NC];
+#pragma unroll
+  for (int i = 0; i < NC; ++i) {
+    const uint32_t pc = (i + rot) & (NC - 1);   // physical chunk held in register slot i
+    const uint32_t *src = cnt32 + tid * WPT + pc * CWD;
+    if constexpr (CWD == 4) {
+      const uint4 x = *reinterpret_cast<const uint4 *>(src);
+      w[i][0] = x.x; w[i][1] = x.y; w[i][2] = x.z; w[i][3] = x.w;
+    } else if constexpr (CWD == 2) {
+      const uint2 x = *reinterpret_cast<const uint2 *>(src);
+      w[i][0] = x.x; w[i][1] = x.y;
+    } else {
+      w[i][0] = src[0];
+    }
+    uint32_t s2 = 0;  // packed (lo-sum, hi-sum), each <= 4096
+#pragma unroll
+    for (int j = 0; j < CWD; ++j) s2 += w[i][j];
+    csum[i] = (s2 & 0xFFFFu) + (s2 >> 16);
+  }
+  uint32_t s = 0;
+#pragma unroll
+  for (int i = 0; i < NC; ++i) s += csum[i];
+  const uint32_t incl = warp_incl_scan(s, lane);
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  uint32_t wpre = 0, tot = 0;
+#pragma unroll
+  for (int i = 0; i < kWarps; ++i) {
+    const uint32_t x = wsum[i];
+    wpre += (i < (int)warp) ? x : 0u;
+    tot += x;
+  }
+  const uint32_t excl = wpre + incl - s;
+  constexpr uint32_t TPR = kThreads >> LOGMP;  // threads per bucket row
+  if ((tid & (TPR - 1)) == 0) rowS[row] = excl;
+  if (tid == 0) rowS[MP] = tot;
+  __syncthreads();
+  // padded run start P_j = S_j + 3j + ((G_j - S_j - 3j) & 3): P_j = G_j (mod 4)
+  // and P_j >= P_{j-1} + h_{j-1}; closed form, no serial dependency over j.
+  const uint32_t Sr = rowS[row];
+  const uint32_t Gr = row < m ? Gj[row] : 0u;
+  const uint32_t pad = 3 * row + ((Gr - Sr - 3 * row) & 3u);
+#pragma unroll
+  for (int i = 0; i < NC; ++i) {
+    const uint32_t pc = (i + rot) & (NC - 1);
+    uint32_t run = excl + pad;  // + sum of the chunks physically before pc
+#pragma unroll
+    for (int i2 = 0; i2 < NC; ++i2) run += (((i2 + rot) & (NC - 1)) < pc) ? csum[i2] : 0u;
+#pragma unroll
+    for (int j = 0; j < CWD; ++j) {
+      const uint32_t x = w[i][j];
+      w[i][j] = run * 0x10001u + (x << 16);      // (run, run + lo)
+      run += (x & 0xFFFFu) + (x >> 16);
+    }
+    uint32_t *dst = cnt32 + tid * WPT + pc * CWD;
+    if constexpr (CWD == 4) *reinterpret_cast<uint4 *>(dst) = make_uint4(w[i][0], w[i][1], w[i][2], w[i][3]);
+    else if constexpr (CWD == 2) *reinterpret_cast<uint2 *>(dst) = make_uint2(w[i][0], w[i][1]);
+    else dst[0] = w[i][0];
+  }
+  if ((tid & (TPR - 1)) == 0) Pj[row] = Sr + pad;
+  bulk_wait_read0();  // keys_s may still be read by this thread's bulk stores of the previous tile
+  __syncthreads();
+
+  // ---- 3. local multisplit of the tile into shared memory
+#pragma unroll
+  for (int q = 0; q < K; ++q) {
+    if (FULL || b0 + q < nt) {
+      uint32_t id;
+      if constexpr (KEEP_ID) id = (idk[q >> 2] >> (8 * (q & 3))) & 255u;
+      else id = id_of(q);
+      const uint32_t slot =
+          *reinterpret_cast<const uint16_t *>(cb + (id << 9)) + ((rk[q >> 3] >> (4 * (q & 7))) & 15u);
+      keys_s[slot] = k[q];
+      if constexpr (KV) vals_s[slot] = v[q];
+    }
+  }
+  fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA (async proxy)
+  __syncthreads();
+
+  // ---- 4. bucket runs: 8 threads per bucket -- 3 head keys, 3 tail keys,
+  //         and the TMA bulk store(s) of the 16-byte-aligned body
+  {
+    const uint32_t b = tid >> 3, sub = tid & 7;
+    if (b < m) {
+      const uint32_t len = rowS[b + 1] - rowS[b];
+      const uint32_t P = Pj[b], Gd = Gj[b];
+      const uint32_t head = min(len, (4u - (Gd & 3u)) & 3u);
+      const uint32_t body = (len - head) & ~3u;
+      if (sub < 6) {
+        const uint32_t i = sub < 3 ? sub : head + body + (sub - 3);
+        if ((sub < 3 && sub < head) || (sub >= 3 && i < len)) {
+          keys_out[Gd + i] = keys_s[P + i];
+          if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+        }
+      } else if (body) {
+        if (sub == 6) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
+        else if (KV) bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
+        bulk_commit();
+      }
+    }
+  }
+}
+
+template <int KIND, bool KV, int LOGMP, bool IDS8>
+__global__ void __launch_bounds__(kThreads, KV ? 2 : 3)
+k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
+             const void *__restrict__ ids, const uint32_t *__restrict__ G,
+             uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
+             uint32_t L, const __grid_constant__ BucketParams p, int reverse) {
+  using Ly = K3pLayout<LOGMP, KV, IDS8>;
+  constexpr int T = Ly::T, STAGES = Ly::STAGES, CW = Ly::CW, MP = Ly::MP;
+  extern __shared__ __align__(128) uint32_t sm[];
+  uint32_t *stk = sm + Ly::O_STK;
+  uint32_t *stv = sm + Ly::O_STV;
+  uint32_t *sti = sm + Ly::O_STI;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t beta = 2 * lane + (warp & 1) + 64 * (warp >> 1);
+  const uint32_t m = p.m;
+  // tiles blockIdx.x, blockIdx.x + gridDim.x, ...; the partial tile (if any)
+  // is the last one overall, hence the last of its CTA: it is peeled off
+  // the loop so its predicated code does not raise the loop's registers.
+  auto tile_of = [&](uint32_t it) -> uint64_t { return (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x; };
+  const uint32_t iters = blockIdx.x < L ? (L - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  const bool has_tail = iters && (uint64_t)n < (uint64_t)L * T && tile_of(iters - 1) == L - 1;
+  const uint32_t iters_full = iters - (has_tail ? 1 : 0);
+
+  if constexpr (KIND == SPLITTERS) {
+    if (tid < (1u << p.logm)) sm[Ly::O_SPL + tid] = p.spl[tid];
+  }
+  // prologue: STAGES tiles in flight
+#pragma unroll
+  for (int s = 0; s < STAGES; ++s) {
+    if ((uint32_t)s < iters) k3p_prefetch<KV, IDS8, T>(stk, stv, sti, s, keys, vals, ids, tile_of(s), n, beta);
+    cp_async_commit();
+  }
+  uint32_t gnext = 0;
+  if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
+
+  // per-iteration prologue: zero the counters (last read by the previous
+  // tile's scatter, before a barrier), publish G[:, tile] into this parity's
+  // metadata, prefetch the next G column, wait for this thread's staged chunks
+  auto begin_tile = [&](uint32_t it, uint32_t *meta) {
+    uint4 *c4 = reinterpret_cast<uint4 *>(sm + Ly::O_CNT);
+#pragma unroll
+    for (int i = 0; i < (CW / 4 + kThreads - 1) / kThreads; ++i) {
+      const int idx = i * kThreads + tid;
+      if (idx < CW / 4) c4[idx] = make_uint4(0, 0, 0, 0);
+    }
+    if (tid < m) meta[MP + 4 + MP + tid] = gnext;
+    if (it + 1 < iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(it + 1));
+    cp_async_wait<STAGES - 1>();
+    __syncthreads();
+  };
+
+  uint32_t it = 0;
+  for (; it < iters_full; ++it) {
+    const uint64_t tile = tile_of(it);
+    const int st = (int)(it % STAGES);
+    uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
+    begin_tile(it, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, true>(stk + st * T, stv + st * T, sti + st * (T / 4), ids, keys_out, vals_out,
+                                          tile * T, T, p, sm, beta, meta);
+    // refill this stage with tile it + STAGES (own chunks only; already consumed)
+    if (it + STAGES < iters)
+      k3p_prefetch<KV, IDS8, T>(stk, stv, sti, st, keys, vals, ids, tile_of(it + STAGES), n, beta);
+    cp_async_commit();
+  }
+  if (has_tail) {
+    const uint64_t tile = tile_of(it);
+    const int st = (int)(it % STAGES);
+    uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
+    begin_tile(it, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, false>(stk + st * T, stv + st * T, sti + st * (T / 4), ids, keys_out,
+                                           vals_out, tile * T, (uint32_t)(n - tile * T), p, sm, beta, meta);
+  }
+  bulk_wait_read0();
+}
+
+}  // namespace ms

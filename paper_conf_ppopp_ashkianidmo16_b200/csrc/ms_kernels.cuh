@@ -13,49 +13,58 @@ namespace ms {
 // Per-tile bucket histogram -> column `tile` of H (bucket-major, H[j*L + l]).
 // Local step 1 of the skeleton, Alg. 1 lines P:819-824.
 //
-// B200 design: 128-bit coalesced loads (KPT keys per thread, all in flight
-// before any use); per-thread PRIVATE packed 8-bit counters in shared memory
-// (column tid of a [ceil(m/4)][256] word array: bank = tid % 32, so the
-// read-modify-write per key never conflicts and needs no atomics); then a
-// CTA reduction of the packed counters (two 16-bit lanes per word).
-// Counters cannot overflow: a thread counts <= KPT <= 32 keys.
+// B200 design: 128-bit streaming loads (KPT keys per thread, all in flight
+// before any use); per-thread PRIVATE byte counters in shared memory,
+// c8[j][slot(tid)] (a thread counts <= KPT <= 32 keys, so a byte never
+// overflows), laid out so the 32 lanes of a warp always hit 32 different
+// banks whatever their bucket ids: 4 instructions per key, no atomics, no
+// warp votes.  Thread j then sums row j (256 bytes) with dp4a, reading
+// 16-byte chunks in a lane-rotated order (conflict-free).
+__device__ __forceinline__ uint32_t k1_slot(uint32_t tid) {
+  const uint32_t lane = tid & 31, warp = tid >> 5;
+  return (warp >> 2) * 128 + lane * 4 + (warp & 3);
+}
+
 template <int KIND, int KPT>
 __global__ void __launch_bounds__(kThreads)
 k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
            uint32_t L, uint32_t *__restrict__ H, const __grid_constant__ BucketParams p,
            uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
   constexpr int T = kThreads * KPT;
+  static_assert(KPT <= 255 && KPT % 4 == 0, "byte counters");
   extern __shared__ __align__(16) uint32_t smem[];
-  uint32_t *spl_s = smem;              // kMaxM words (SPLITTERS)
-  uint32_t *cnt = smem + kMaxM;        // [nwords][256]
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  uint32_t *spl_s = smem;                                     // kMaxM words (SPLITTERS)
+  uint8_t *c8 = reinterpret_cast<uint8_t *>(smem + kMaxM);    // [m][256] bytes
+  const uint32_t tid = threadIdx.x, lane = tid & 31;
   const uint32_t tile = blockIdx.x;
   const uint64_t base = (uint64_t)tile * T;
   const uint32_t nt = (uint32_t)umin64(T, n - base);
-  const uint32_t nwords = (p.m + 3) >> 2;
+  const uint32_t m = p.m;
 
+  // issue this thread's loads first (they overlap the shared-memory setup)
+  uint4 v[KPT / 4];
+  const bool full = (nt == T);
+  if (full) {
+    const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
+#pragma unroll
+    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldcs(k4 + j * kThreads + tid);
+  }
   // K2's look-back status words are cleared here (K1 precedes K2 in the stream).
   for (uint32_t i = tile * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
-  for (uint32_t i = tid; i < nwords * kThreads; i += kThreads) cnt[i] = 0;
+  uint4 *c4 = reinterpret_cast<uint4 *>(c8);
+  for (uint32_t i = tid; i < m * 16; i += kThreads) c4[i] = make_uint4(0, 0, 0, 0);
   if constexpr (KIND == SPLITTERS) {
     for (uint32_t i = tid; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
   }
   __syncthreads();
 
+  uint8_t *mine = c8 + k1_slot(tid);
   uint32_t bad = 0;
-  auto count = [&](uint32_t id) {
-    uint32_t *c = cnt + (id >> 2) * kThreads + tid;
-    *c += 1u << ((id & 3u) * 8u);
-  };
-  if (nt == T) {
-    const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
-    uint4 v[KPT / 4];
-#pragma unroll
-    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldcs(k4 + j * kThreads + tid);  // streaming
+  if (full) {
     if constexpr (KIND == IDS) {
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) {
-        uint64_t i0 = base + 4ull * (j * kThreads + tid);
+        const uint64_t i0 = base + 4ull * (j * kThreads + tid);
         uint32_t raw[4];
         if (p.id_bytes == 1) {
           uint32_t w = __ldg(reinterpret_cast<const uint32_t *>((const uint8_t *)ids + i0));
@@ -67,16 +76,16 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
           bad |= raw[q] > p.mmask;
-          count(min(raw[q], p.mmask));
+          mine[min(raw[q], p.mmask) * kThreads] += 1;
         }
       }
     } else {
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) {
-        count(bucket_of_key<KIND>(v[j].x, p, spl_s));
-        count(bucket_of_key<KIND>(v[j].y, p, spl_s));
-        count(bucket_of_key<KIND>(v[j].z, p, spl_s));
-        count(bucket_of_key<KIND>(v[j].w, p, spl_s));
+        mine[bucket_of_key<KIND>(v[j].x, p, spl_s) * kThreads] += 1;
+        mine[bucket_of_key<KIND>(v[j].y, p, spl_s) * kThreads] += 1;
+        mine[bucket_of_key<KIND>(v[j].z, p, spl_s) * kThreads] += 1;
+        mine[bucket_of_key<KIND>(v[j].w, p, spl_s) * kThreads] += 1;
       }
     }
   } else {
@@ -90,7 +99,7 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
       } else {
         id = bucket_of_key<KIND>(keys[base + i], p, spl_s);
       }
-      count(id);
+      mine[id * kThreads] += 1;
     }
   }
   if constexpr (KIND == IDS) {
@@ -98,23 +107,19 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   }
   __syncthreads();
 
-  // CTA reduction of the packed counters: warp w owns words w, w+8, ...
-  for (uint32_t q = warp; q < nwords; q += kWarps) {
-    uint32_t lo = 0, hi = 0;
+  // row j = bucket j's 256 byte counters; thread j sums it
+  if (tid < m) {
+    const uint4 *row = c4 + tid * 16;
+    uint32_t acc = 0;
 #pragma unroll
-    for (int j = 0; j < kThreads / 32; ++j) {
-      uint32_t x = cnt[q * kThreads + j * 32 + lane];
-      lo += x & 0x00FF00FFu;
-      hi += (x >> 8) & 0x00FF00FFu;
+    for (int j = 0; j < 16; ++j) {
+      const uint4 w = row[(j + tid) & 15];
+      acc = __dp4a(w.x, 0x01010101u, acc);
+      acc = __dp4a(w.y, 0x01010101u, acc);
+      acc = __dp4a(w.z, 0x01010101u, acc);
+      acc = __dp4a(w.w, 0x01010101u, acc);
     }
-    lo = warp_sum(lo);
-    hi = warp_sum(hi);
-    if (lane < 4) {
-      uint32_t b = 4 * q + lane;
-      uint32_t c = lane == 0 ? (lo & 0xFFFFu) : lane == 1 ? (hi & 0xFFFFu)
-                 : lane == 2 ? (lo >> 16) : (hi >> 16);
-      if (b < p.m) H[(uint64_t)b * L + tile] = c;
-    }
+    H[(uint64_t)tid * L + tile] = acc;
   }
 }
 
@@ -229,13 +234,118 @@ k2_scan(uint32_t *__restrict__ data, uint64_t total, uint64_t *__restrict__ stat
 // Tile = 8 warps x R rounds x 32 keys; warp w owns the contiguous segment
 // [w*32R, (w+1)*32R) and walks it in rounds of 32 consecutive keys, so
 // (warp, round, lane) order IS input order and ranks are stable.
-// Per round: logm ballots give each lane the mask of same-bucket lanes
-// (Alg. 3 with the exclusive-rank fix, reading #4); the highest
-// lane of each bucket group advances the warp's smem counter (Alg. 2's
-// histogram, accumulated).  Cross-warp exclusive prefixes + the tile's
-// bucket starts S_t then give each key its shared-memory slot (Eq. (2)
-// applied one level down).
-// Keys (and values) arrive by one TMA bulk copy per array (UBLKCP).
+// Per round one __match_any_sync gives each lane the mask of same-bucket
+// lanes (the role of Alg. 3's log m ballots; measured ~6x cheaper on sm_100
+// at m = 32), popc(mask & lanemask_lt) is the exclusive rank
+// (reading #4), and the highest lane of each group advances the warp's
+// shared-memory counter for that bucket.  Cross-warp exclusive prefixes +
+// the tile's bucket starts S_t then give each key its shared-memory slot
+// (Eq. (2) one level down).  Keys (and values) arrive by one TMA
+// bulk copy per array (UBLKCP) on an mbarrier.
+template <int KIND, bool KV, int R, bool FULL>
+__device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
+                                        uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
+                                        uint64_t base, uint32_t nt, const BucketParams &p,
+                                        uint32_t *keys_s, uint32_t *vals_s, uint32_t *cnt_s,
+                                        uint32_t *gD_s, const uint32_t *spl_s, uint8_t *id8_s,
+                                        uint32_t *wsum, uint32_t gcol) {
+  constexpr int SEG = 32 * R;
+  constexpr bool ID8 = (KIND != LOWBITS && KIND != SHIFTC);
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t m = p.m;
+  const uint32_t lt = lanemask_lt(), gt = lanemask_gt();
+  uint32_t *cnt_w = cnt_s + warp * kMaxM;
+  const uint32_t seg0 = warp * SEG + lane;
+
+  uint32_t idr[KIND == IDS ? R : 1];
+  if constexpr (KIND == IDS) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint32_t pos = seg0 + r * 32;
+      idr[r] = (FULL || pos < nt) ? load_id(ids, base + pos, p) : 0xFFFFFFFFu;
+    }
+  }
+
+  // ---- phase 1: stable ranks within the warp's segment
+  uint32_t kreg[R];
+  uint32_t vreg[KV ? R : 1];
+  uint32_t pk[R];  // (rank within warp segment) << 8 | id
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t pos = seg0 + r * 32;
+    const bool valid = FULL || pos < nt;
+    const uint32_t key = keys_s[pos];
+    uint32_t id;
+    if constexpr (KIND == IDS) id = idr[r];
+    else id = valid ? bucket_of_key<KIND>(key, p, spl_s) : 0xFFFFFFFFu;
+    const uint32_t peers = __match_any_sync(0xFFFFFFFFu, id);
+    const uint32_t rank = __popc(peers & lt);
+    uint32_t before = 0;
+    if (valid) before = cnt_w[id];
+    __syncwarp();
+    if (valid && (peers & gt) == 0) cnt_w[id] = before + __popc(peers);
+    __syncwarp();
+    kreg[r] = key;
+    if constexpr (KV) vreg[r] = vals_s[pos];
+    pk[r] = ((before + rank) << 8) | (id & 255u);
+  }
+  __syncthreads();
+
+  // ---- per-bucket cross-warp exclusive prefix, tile bucket starts S_t
+  uint32_t tot = 0;
+  if (tid < m) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) {
+      const uint32_t c = cnt_s[w * kMaxM + tid];
+      cnt_s[w * kMaxM + tid] = tot;
+      tot += c;
+    }
+  }
+  const uint32_t incl = warp_incl_scan(tot, lane);
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  uint32_t wpre = 0;
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) wpre += (w < (int)warp) ? wsum[w] : 0u;
+  const uint32_t S = wpre + incl - tot;  // exclusive scan of the tile histogram
+  if (tid < m) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] += S;
+    gD_s[tid] = gcol - S;
+  }
+  __syncthreads();
+
+  // ---- local multisplit of the tile into shared memory (in place)
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (FULL || seg0 + r * 32 < nt) {
+      const uint32_t id = pk[r] & 255u;
+      const uint32_t slot = cnt_w[id] + (pk[r] >> 8);
+      keys_s[slot] = kreg[r];
+      if constexpr (KV) vals_s[slot] = vreg[r];
+      if constexpr (ID8) id8_s[slot] = (uint8_t)id;
+    }
+  }
+  __syncthreads();
+
+  // ---- coalesced stores of the bucket runs
+  auto store = [&](uint32_t i) {
+    const uint32_t k = keys_s[i];
+    uint32_t id;
+    if constexpr (ID8) id = id8_s[i];
+    else id = bucket_of_key<KIND>(k, p, spl_s);
+    const uint32_t dst = gD_s[id] + i;
+    __stcs(keys_out + dst, k);
+    if constexpr (KV) __stcs(vals_out + dst, vals_s[i]);
+  };
+  if constexpr (FULL) {
+#pragma unroll 4
+    for (int j = 0; j < R; ++j) store(j * kThreads + tid);
+  } else {
+    for (uint32_t i = tid; i < nt; i += kThreads) store(i);
+  }
+}
+
 template <int KIND, bool KV, int R>
 __global__ void __launch_bounds__(kThreads)
 k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
@@ -243,8 +353,6 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
             uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
             uint32_t L, const __grid_constant__ BucketParams p) {
   constexpr int T = kThreads * R;
-  constexpr int SEG = 32 * R;
-  constexpr bool NEED_ID8 = (KIND == SPLITTERS || KIND == IDS);
   extern __shared__ __align__(128) uint8_t smem_raw[];
   uint32_t *keys_s = reinterpret_cast<uint32_t *>(smem_raw);
   uint32_t *vals_s = keys_s + T;
@@ -255,7 +363,7 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   __shared__ __align__(8) uint64_t bar;
   __shared__ uint32_t wsum[kWarps];
 
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t tid = threadIdx.x;
   const uint32_t tile = blockIdx.x;
   const uint64_t base = (uint64_t)tile * T;
   const uint32_t nt = (uint32_t)umin64(T, n - base);
@@ -285,92 +393,13 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
     if (tid < (1u << p.logm)) spl_s[tid] = p.spl[tid];
   }
   __syncthreads();
-  if (full) mbar_wait(&bar, 0);
-
-  // ---- phase 1: stable ranks within the warp's segment
-  const uint32_t lt = lanemask_lt();
-  uint32_t kreg[R];
-  uint32_t vreg[KV ? R : 1];
-  uint32_t pk[R];  // (rank within warp segment) << 8 | id
-  uint32_t *cnt_w = cnt_s + warp * kMaxM;
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    const uint32_t pos = warp * SEG + r * 32 + lane;
-    const bool valid = full || pos < nt;
-    const uint32_t key = keys_s[pos];
-    uint32_t id = 0;
-    if (valid) {
-      if constexpr (KIND == IDS) id = load_id(ids, base + pos, p);
-      else id = bucket_of_key<KIND>(key, p, spl_s);
-    }
-    uint32_t peers = full ? 0xFFFFFFFFu : __ballot_sync(0xFFFFFFFFu, valid);
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      if ((uint32_t)k < p.logm) {
-        const uint32_t bit = (id >> k) & 1u;
-        const uint32_t b = __ballot_sync(0xFFFFFFFFu, bit);
-        peers &= bit ? b : ~b;
-      }
-    }
-    const uint32_t rank = __popc(peers & lt);
-    uint32_t before = 0;
-    if (valid) before = cnt_w[id];
-    __syncwarp();
-    if (valid && (peers >> lane) == 1u) cnt_w[id] = before + __popc(peers);
-    __syncwarp();
-    kreg[r] = key;
-    if constexpr (KV) vreg[r] = vals_s[pos];
-    pk[r] = ((before + rank) << 8) | id;
-  }
-  __syncthreads();
-
-  // ---- per-bucket cross-warp exclusive prefix, tile bucket starts S_t
-  uint32_t tot = 0;
-  if (tid < m) {
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) {
-      uint32_t c = cnt_s[w * kMaxM + tid];
-      cnt_s[w * kMaxM + tid] = tot;
-      tot += c;
-    }
-  }
-  const uint32_t incl = warp_incl_scan(tot, lane);
-  if (lane == 31) wsum[warp] = incl;
-  __syncthreads();
-  uint32_t wpre = 0;
-#pragma unroll
-  for (int w = 0; w < kWarps; ++w) wpre += (w < (int)warp) ? wsum[w] : 0u;
-  const uint32_t S = wpre + incl - tot;  // exclusive scan of tile histogram
-  if (tid < m) {
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] += S;
-    gD_s[tid] = gcol - S;
-  }
-  __syncthreads();
-
-  // ---- local multisplit of the tile into shared memory
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    const uint32_t pos = warp * SEG + r * 32 + lane;
-    if (full || pos < nt) {
-      const uint32_t id = pk[r] & 255u;
-      const uint32_t slot = cnt_w[id] + (pk[r] >> 8);
-      keys_s[slot] = kreg[r];
-      if constexpr (KV) vals_s[slot] = vreg[r];
-      if constexpr (NEED_ID8) id8_s[slot] = (uint8_t)id;
-    }
-  }
-  __syncthreads();
-
-  // ---- coalesced stores of the bucket runs
-  for (uint32_t i = tid; i < nt; i += kThreads) {
-    const uint32_t k = keys_s[i];
-    uint32_t id;
-    if constexpr (NEED_ID8) id = id8_s[i];
-    else id = bucket_of_key<KIND>(k, p, spl_s);
-    const uint32_t dst = gD_s[id] + i;
-    __stcs(keys_out + dst, k);
-    if constexpr (KV) __stcs(vals_out + dst, vals_s[i]);
+  if (full) {
+    mbar_wait(&bar, 0);
+    k3_tile<KIND, KV, R, true>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+                               spl_s, id8_s, wsum, gcol);
+  } else {
+    k3_tile<KIND, KV, R, false>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+                                spl_s, id8_s, wsum, gcol);
   }
 }
 
