@@ -15,7 +15,7 @@
 
 #include "../../include/ms.h"
 #include "ms_kernels.cuh"
-#include "ms_k3_blocked.cuh"
+#include "ms_k3p_args.h"
 
 using namespace ms;
 
@@ -26,7 +26,7 @@ struct ms_plan_s {
   uint32_t flags;
   BucketParams bp;
   int kkind;  // kernel-level Kind (ms_device.cuh)
-  int reverse = 0;  // K3 walks tiles last-to-first (L2 reuse of K1's tail)
+  uint32_t kpt = 16;  // K3 (m <= 32): keys per thread, tile T = 256 * kpt
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
   int tracing = 0;
@@ -68,8 +68,8 @@ uint64_t delta_magic(uint32_t d) { return ~0ull / d + 1; }
 // Rounds per warp R (tile T = 256 R): 16 for m <= 32, 32 above (runs of T/m
 // keys stay >= 32 keys = 128 B); halved while the grid would not fill two
 // waves of 148 SMs (small n is launch/latency bound, not HBM bound).
-int rounds_for(uint32_t m, uint64_t n) {
-  if (m <= 32) return 16;  // K3b (blocked ranks) uses T = 4096 for every n
+int rounds_for(uint32_t m, uint64_t n, uint32_t kpt) {
+  if (m <= 32) return (int)kpt;  // blocked-rank K3: T = 256 * kpt for every n
   int R = 16;
   while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
   return R;
@@ -86,7 +86,7 @@ struct Geometry {
 
 Geometry geometry(const ms_plan_s *p, uint64_t n) {
   Geometry g{};
-  g.R = rounds_for(p->spec.m, n);
+  g.R = rounds_for(p->spec.m, n, p->kpt);
   g.T = 256u * g.R;
   g.L = (n + g.T - 1) / g.T;
   g.hg_words = (uint64_t)p->spec.m * g.L;
@@ -174,9 +174,7 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   }
 }
 
-// Persistent grid: SM count x resident CTAs per SM (cached per kernel).
-template <typename K>
-unsigned persistent_grid(K kernel, size_t smem, uint64_t tiles) {
+int sm_count() {
   static int sms = 0;
   if (!sms) {
     int dev = 0;
@@ -184,61 +182,23 @@ unsigned persistent_grid(K kernel, size_t smem, uint64_t tiles) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     if (sms <= 0) sms = 148;
   }
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kThreads, smem);
-  if (per_sm <= 0) per_sm = 1;
-  return (unsigned)std::min<uint64_t>(tiles, (uint64_t)sms * per_sm);
-}
-
-template <int KIND, bool KV, int LOGMP>
-cudaError_t launch_k3b_l(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const uint32_t *vals,
-                         const void *ids, const uint32_t *G, uint32_t *ko, uint32_t *vo, uint32_t n,
-                         cudaStream_t s) {
-  if (KIND == IDS && p->spec.id_bytes == 1) {
-    auto k = k3p_postscan<KIND, KV, LOGMP, true>;
-    const size_t smem = K3pLayout<LOGMP, KV, true>::BYTES;
-    set_smem(k, smem);
-    k<<<persistent_grid(k, smem, g.L), kThreads, smem, s>>>(keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->bp,
-                                                           p->reverse);
-  } else {
-    auto k = k3p_postscan<KIND, KV, LOGMP, false>;
-    const size_t smem = K3pLayout<LOGMP, KV, false>::BYTES;
-    set_smem(k, smem);
-    k<<<persistent_grid(k, smem, g.L), kThreads, smem, s>>>(keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->bp,
-                                                           p->reverse);
-  }
-  return cudaGetLastError();
-}
-
-template <int KIND, bool KV>
-cudaError_t launch_k3b(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const uint32_t *vals,
-                       const void *ids, const uint32_t *G, uint32_t *ko, uint32_t *vo, uint32_t n,
-                       cudaStream_t s) {
-  switch (std::max<uint32_t>(1, ceil_log2(p->spec.m))) {
-    case 1: return launch_k3b_l<KIND, KV, 1>(p, g, keys, vals, ids, G, ko, vo, n, s);
-    case 2: return launch_k3b_l<KIND, KV, 2>(p, g, keys, vals, ids, G, ko, vo, n, s);
-    case 3: return launch_k3b_l<KIND, KV, 3>(p, g, keys, vals, ids, G, ko, vo, n, s);
-    case 4: return launch_k3b_l<KIND, KV, 4>(p, g, keys, vals, ids, G, ko, vo, n, s);
-    default: return launch_k3b_l<KIND, KV, 5>(p, g, keys, vals, ids, G, ko, vo, n, s);
-  }
+  return sms;
 }
 
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                         uint32_t *vo, uint32_t n, cudaStream_t s) {
   const bool kv = vals != nullptr;
-  if (p->spec.m <= 32) {
-#define MS_K3B(KIND)                                                        \
-  return kv ? launch_k3b<KIND, true>(p, g, keys, vals, ids, G, ko, vo, n, s) \
-            : launch_k3b<KIND, false>(p, g, keys, vals, ids, G, ko, vo, n, s);
+  if (p->spec.m <= 32) {  // persistent blocked-rank K3 (ms_k3_blocked.cuh), one TU per kind
+    K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes, p->kpt, &p->bp,
+              sm_count(), s};
     switch (p->kkind) {
-      case LOWBITS: MS_K3B(LOWBITS)
-      case SHIFTC: MS_K3B(SHIFTC)
-      case DELTA: MS_K3B(DELTA)
-      case SPLITTERS: MS_K3B(SPLITTERS)
-      default: MS_K3B(IDS)
+      case LOWBITS: return k3p_launch_lowbits(a);
+      case SHIFTC: return k3p_launch_shiftc(a);
+      case DELTA: return k3p_launch_delta(a);
+      case SPLITTERS: return k3p_launch_splitters(a);
+      default: return k3p_launch_ids(a);
     }
-#undef MS_K3B
   }
 #define MS_K3K(KIND)                                                     \
   return kv ? launch_k3<KIND, true>(p, g, keys, vals, ids, G, ko, vo, n, s) \
@@ -347,8 +307,9 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->bp = bp;
   p->kkind = kkind;
   p->last_launches = 0;
-  // ablation override: MS_K3_REVERSE=1 makes K3 walk tiles last-to-first
-  if (const char *e = getenv("MS_K3_REVERSE")) p->reverse = atoi(e) ? 1 : 0;
+  // ablation override: MS_K3_KPT=16|32 keys per thread in K3 (m <= 32)
+  if (const char *e = getenv("MS_K3_KPT")) p->kpt = atoi(e) == 32 ? 32u : 16u;
+  if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
   *plan = p;
   return MS_OK;
 }

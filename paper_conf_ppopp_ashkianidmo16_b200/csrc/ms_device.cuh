@@ -29,6 +29,7 @@ struct BucketParams {
   uint32_t logm;      // ceil(log2 m): splitter search steps
   uint32_t id_bytes;  // IDS: 1 or 4
   uint32_t validate;  // IDS: flag ids >= m
+  uint32_t dbg;       // ablation switch (MS_DEBUG_K3): 0 normal
   uint32_t spl[kMaxM];
 };
 
@@ -147,6 +148,7 @@ __device__ __forceinline__ void bulk_wait_read0() {
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+inline uint64_t umin64_host(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t r;

@@ -26,18 +26,22 @@
 // prefetches its own next blocks with cp.async (LDGSTS) into a chunk-major
 // staging ring, so loads for the next STAGES tiles are in flight while the
 // current tile is ranked and stored, and no barrier guards the staging data.
+#include "ms_k3p_args.h"
+
 namespace ms {
 
-template <int LOGMP, bool KV, bool IDS8>
+template <int LOGMP, bool KV, bool IDS8, int KPT>
 struct K3pLayout {
   static constexpr int MP = 1 << LOGMP;        // bucket rows (m rounded up to a power of 2, >= 2)
-  static constexpr int K = 16;                 // keys per thread
-  static constexpr int T = kThreads * K;       // 4096 keys per tile
-  static constexpr int STAGES = KV ? 1 : 2;    // tiles prefetched ahead
+  static constexpr int K = KPT;                // keys per thread (16 or 32)
+  static constexpr int CH = K / 4;             // 16-byte chunks per thread per array
+  static constexpr int T = kThreads * K;       // keys per tile
+  static constexpr int STAGES = (KV || K > 16) ? 1 : 2;  // tiles prefetched ahead
   static constexpr int CW = MP * 128;          // counter words (MP x 256 u16)
   static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // key slots incl. alignment padding
   static constexpr int WPT = MP / 2;           // counter words per thread in the scan
   static constexpr int MW = 3 * MP + 8;        // per-tile metadata words: rowS[MP+4] P[MP] G[MP]
+  static constexpr int IW = IDS8 ? T / 4 : 0;  // staged u8 ids per stage (words)
   // word offsets
   static constexpr int O_CNT = 0;
   static constexpr int O_KEYS = O_CNT + CW;
@@ -45,7 +49,7 @@ struct K3pLayout {
   static constexpr int O_STK = O_VALS + (KV ? KSR : 0);           // [STAGES][T] keys
   static constexpr int O_STV = O_STK + STAGES * T;                // [STAGES][T] vals
   static constexpr int O_STI = O_STV + (KV ? STAGES * T : 0);     // [STAGES][T/4] u8 ids
-  static constexpr int O_META = O_STI + (IDS8 ? STAGES * T / 4 : 0);  // [2][MW] (tile parity)
+  static constexpr int O_META = O_STI + STAGES * IW;              // [2][MW] (tile parity)
   static constexpr int O_WS = O_META + 2 * MW;
   static constexpr int O_SPL = O_WS + 12;
   static constexpr int WORDS = O_SPL + kMaxM;
@@ -66,27 +70,32 @@ __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
 
-// Stage this thread's chunks of tile `tile` (keys: 4 x 16 B; vals likewise;
-// u8 ids: 1 x 16 B) into stage slot `st`, chunk-major ([c][tid]) so the
+// Stage this thread's chunks of tile `tile` (keys: CH x 16 B; vals likewise;
+// u8 ids: K/16 x 16 B) into stage slot `st`, chunk-major ([c][tid]) so the
 // later 128-bit reads are conflict-free.  Bytes past n are zero-filled.
-template <bool KV, bool IDS8, int T>
+template <bool KV, bool IDS8, int T, int K>
 __device__ __forceinline__ void k3p_prefetch(uint32_t *stk, uint32_t *stv, uint32_t *sti, int st,
                                              const uint32_t *keys, const uint32_t *vals, const void *ids,
                                              uint64_t tile, uint32_t n, uint32_t beta) {
+  constexpr int CH = K / 4;
   const uint32_t tid = threadIdx.x;
-  const uint64_t b0 = tile * T + beta * 16ull;
+  const uint64_t b0 = tile * T + (uint64_t)beta * K;
   uint32_t *dk = stk + st * T + tid * 4;
   uint32_t *dv = stv + st * T + tid * 4;
+  uint32_t *di = sti + st * (T / 4) + tid * 4;
   if (tile * T + T <= n) {
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
+    for (int c = 0; c < CH; ++c) {
       cp_async16_full(dk + c * kThreads * 4, keys + b0 + 4 * c);
       if constexpr (KV) cp_async16_full(dv + c * kThreads * 4, vals + b0 + 4 * c);
     }
-    if constexpr (IDS8) cp_async16_full(sti + st * (T / 4) + tid * 4, (const uint8_t *)ids + b0);
+    if constexpr (IDS8) {
+#pragma unroll
+      for (int c = 0; c < K / 16; ++c) cp_async16_full(di + c * kThreads * 4, (const uint8_t *)ids + b0 + 16 * c);
+    }
   } else {
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
+    for (int c = 0; c < CH; ++c) {
       const uint64_t e = b0 + 4 * c;
       const uint32_t bytes = e >= n ? 0u : (uint32_t)(umin64(4, n - e) * 4);
       const uint64_t src = bytes ? e : 0;
@@ -94,20 +103,24 @@ __device__ __forceinline__ void k3p_prefetch(uint32_t *stk, uint32_t *stv, uint3
       if constexpr (KV) cp_async16(dv + c * kThreads * 4, vals + src, bytes);
     }
     if constexpr (IDS8) {
-      const uint32_t bytes = b0 >= n ? 0u : (uint32_t)umin64(16, n - b0);
-      cp_async16(sti + st * (T / 4) + tid * 4, (const uint8_t *)ids + (bytes ? b0 : 0), bytes);
+#pragma unroll
+      for (int c = 0; c < K / 16; ++c) {
+        const uint64_t e = b0 + 16 * c;
+        const uint32_t bytes = e >= n ? 0u : (uint32_t)umin64(16, n - e);
+        cp_async16(di + c * kThreads * 4, (const uint8_t *)ids + (bytes ? e : 0), bytes);
+      }
     }
   }
 }
 
-// One tile, already staged.  FULL: all 4096 keys valid (no per-key predicates).
-template <int KIND, bool KV, int LOGMP, bool IDS8, bool FULL>
+// One tile, already staged.  FULL: all T keys valid (no per-key predicates).
+template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, bool FULL>
 __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *sm_v, const uint32_t *sm_i,
                                          const void *__restrict__ ids, uint32_t *__restrict__ keys_out,
                                          uint32_t *__restrict__ vals_out, uint64_t base, uint32_t nt,
                                          const BucketParams &p, uint32_t *sm, uint32_t beta, uint32_t *meta) {
-  using Ly = K3pLayout<LOGMP, KV, IDS8>;
-  constexpr int MP = Ly::MP, K = Ly::K;
+  using Ly = K3pLayout<LOGMP, KV, IDS8, KPT>;
+  constexpr int MP = Ly::MP, K = Ly::K, CH = Ly::CH;
   // ids are recomputed from the key where that is cheaper than keeping them
   constexpr bool KEEP_ID = (KIND == SPLITTERS) || (KIND == IDS && !IDS8);
   uint32_t *cnt32 = sm + Ly::O_CNT;
@@ -124,45 +137,64 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   // this thread's counter column: byte address of c[0][beta]; c[j][beta] is j*512 bytes further
   uint8_t *cb = reinterpret_cast<uint8_t *>(cnt32) + 2 * beta;
 
-  // ---- own staged chunks -> registers
-  uint32_t k[K];
-  uint32_t v[KV ? K : 1];
+  // Keys (and values) are read from this thread's own staged chunks twice --
+  // for counting and again for the scatter -- instead of being held in
+  // registers across the scan (no spills at 3 CTAs/SM).
+  auto chunk = [&](const uint32_t *st, int c) -> uint4 {
+    return *reinterpret_cast<const uint4 *>(st + (c * kThreads + tid) * 4);
+  };
+  uint32_t idw[IDS8 ? K / 4 : 1];
+  if constexpr (IDS8) {
 #pragma unroll
-  for (int c = 0; c < 4; ++c) {
-    const uint4 x = *reinterpret_cast<const uint4 *>(sm_k + (c * kThreads + tid) * 4);
-    k[4 * c] = x.x; k[4 * c + 1] = x.y; k[4 * c + 2] = x.z; k[4 * c + 3] = x.w;
-    if constexpr (KV) {
-      const uint4 y = *reinterpret_cast<const uint4 *>(sm_v + (c * kThreads + tid) * 4);
-      v[4 * c] = y.x; v[4 * c + 1] = y.y; v[4 * c + 2] = y.z; v[4 * c + 3] = y.w;
+    for (int c = 0; c < K / 16; ++c) {
+      const uint4 x = chunk(sm_i, c);
+      idw[4 * c] = x.x; idw[4 * c + 1] = x.y; idw[4 * c + 2] = x.z; idw[4 * c + 3] = x.w;
     }
   }
-  uint32_t idw[IDS8 ? 4 : 1];
-  if constexpr (IDS8) {
-    const uint4 x = *reinterpret_cast<const uint4 *>(sm_i + tid * 4);
-    idw[0] = x.x; idw[1] = x.y; idw[2] = x.z; idw[3] = x.w;
-  }
-  auto id_of = [&](int q) -> uint32_t {
+  auto id_of = [&](uint32_t key, int q) -> uint32_t {
     if constexpr (KIND == IDS) {
-      if constexpr (IDS8) return min((idw[q >> 2] >> (8 * (q & 3))) & 255u, p.mmask);
+      if constexpr (IDS8) return min(__byte_perm(idw[q >> 2], 0u, 0x4440u + (q & 3)), p.mmask);
       else return (FULL || b0 + q < nt) ? load_id(ids, base + b0 + q, p) : 0u;
     } else {
-      return bucket_of_key<KIND>(k[q], p, spl_s);
+      return bucket_of_key<KIND>(key, p, spl_s);
     }
   };
 
-  // ---- 1. sequential per-block counting: the rank within the block
-  uint32_t rk[2] = {0u, 0u};                 // 4-bit ranks (< 16), 8 per word
-  uint32_t idk[KEEP_ID ? 4 : 1];             // kept ids, 8 bits each
-  if constexpr (KEEP_ID) idk[0] = idk[1] = idk[2] = idk[3] = 0u;
+  // ---- 1. sequential per-block counting: the rank within the block.
+  // Groups of 4 keys (one staged chunk): the 4 counter loads are issued
+  // together and equal ids inside the group are corrected by compares, so
+  // the read-modify-write chain through shared memory is 4 keys deep
+  // instead of 1.  Keys past the tail (partial tile only) are skipped.
+  uint32_t rk[K / 4];                        // ranks (< K), one byte each
+  uint32_t idk[KEEP_ID ? K / 4 : 1];         // kept ids, one byte each
+  uint4 kx[CH];  // all staged chunks first: no chunk load waits behind a counter store
 #pragma unroll
-  for (int q = 0; q < K; ++q) {
-    const uint32_t id = id_of(q);
-    if (FULL || b0 + q < nt) {
-      uint16_t *c = reinterpret_cast<uint16_t *>(cb + (id << 9));
-      const uint32_t r = *c;
-      *c = (uint16_t)(r + 1);
-      rk[q >> 3] += r << (4 * (q & 7));
-      if constexpr (KEEP_ID) idk[q >> 2] |= id << (8 * (q & 3));
+  for (int c = 0; c < CH; ++c) kx[c] = chunk(sm_k, c);
+#pragma unroll
+  for (int c = 0; c < CH; ++c) {
+    const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
+    uint32_t id[4], r[4];
+    bool ok[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      id[j] = id_of(kk[j], 4 * c + j);
+      ok[j] = FULL || (b0 + 4 * c + j < nt);
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) r[j] = ok[j] ? *reinterpret_cast<const uint16_t *>(cb + (id[j] << 9)) : 0u;
+#pragma unroll
+    for (int j = 1; j < 4; ++j)
+#pragma unroll
+      for (int i = 0; i < j; ++i) r[j] += (ok[i] && id[i] == id[j]) ? 1u : 0u;
+    rk[c] = 0u;
+    if constexpr (KEEP_ID) idk[c] = 0u;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if (ok[j]) {
+        *reinterpret_cast<uint16_t *>(cb + (id[j] << 9)) = (uint16_t)(r[j] + 1);
+        rk[c] |= r[j] << (8 * j);
+        if constexpr (KEEP_ID) idk[c] |= id[j] << (8 * j);
+      }
     }
   }
   __syncthreads();
@@ -191,7 +223,7 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
     } else {
       w[i][0] = src[0];
     }
-    uint32_t s2 = 0;  // packed (lo-sum, hi-sum), each <= 4096
+    uint32_t s2 = 0;  // packed (lo-sum, hi-sum), each <= T/2 + ... < 2^16
 #pragma unroll
     for (int j = 0; j < CWD; ++j) s2 += w[i][j];
     csum[i] = (s2 & 0xFFFFu) + (s2 >> 16);
@@ -211,12 +243,21 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   }
   const uint32_t excl = wpre + incl - s;
   constexpr uint32_t TPR = kThreads >> LOGMP;  // threads per bucket row
+  // S_row = excl of the row's first thread: a lane of this warp (rows < 32
+  // threads) or lane 0 of warp row*TPR/32, whose excl is the warp prefix.
+  uint32_t Sr;
+  if constexpr (TPR < 32) {
+    Sr = __shfl_sync(0xFFFFFFFFu, excl, lane & ~(TPR - 1));
+  } else {
+    Sr = 0;
+    const uint32_t w0 = (row * TPR) >> 5;
+#pragma unroll
+    for (int i = 0; i < kWarps; ++i) Sr += ((uint32_t)i < w0) ? wsum[i] : 0u;
+  }
   if ((tid & (TPR - 1)) == 0) rowS[row] = excl;
   if (tid == 0) rowS[MP] = tot;
-  __syncthreads();
   // padded run start P_j = S_j + 3j + ((G_j - S_j - 3j) & 3): P_j = G_j (mod 4)
   // and P_j >= P_{j-1} + h_{j-1}; closed form, no serial dependency over j.
-  const uint32_t Sr = rowS[row];
   const uint32_t Gr = row < m ? Gj[row] : 0u;
   const uint32_t pad = 3 * row + ((Gr - Sr - 3 * row) & 3u);
 #pragma unroll
@@ -240,17 +281,39 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   bulk_wait_read0();  // keys_s may still be read by this thread's bulk stores of the previous tile
   __syncthreads();
 
-  // ---- 3. local multisplit of the tile into shared memory
+  // ---- 3. local multisplit of the tile into shared memory, one staged
+  // chunk (4 keys) at a time: its 4 slot bases are loaded before its stores
+  uint4 sx[CH];  // staged keys (and values) first, then the per-chunk slot loads and stores
+  uint4 sy[KV ? CH : 1];
 #pragma unroll
-  for (int q = 0; q < K; ++q) {
-    if (FULL || b0 + q < nt) {
+  for (int c = 0; c < CH; ++c) {
+    sx[c] = chunk(sm_k, c);
+    if constexpr (KV) sy[c] = chunk(sm_v, c);
+  }
+#pragma unroll
+  for (int c = 0; c < CH; ++c) {
+    const uint32_t kk[4] = {sx[c].x, sx[c].y, sx[c].z, sx[c].w};
+    uint32_t vv[4];
+    if constexpr (KV) {
+      vv[0] = sy[c].x; vv[1] = sy[c].y; vv[2] = sy[c].z; vv[3] = sy[c].w;
+    }
+    uint32_t sl[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int q = 4 * c + j;
       uint32_t id;
-      if constexpr (KEEP_ID) id = (idk[q >> 2] >> (8 * (q & 3))) & 255u;
-      else id = id_of(q);
-      const uint32_t slot =
-          *reinterpret_cast<const uint16_t *>(cb + (id << 9)) + ((rk[q >> 3] >> (4 * (q & 7))) & 15u);
-      keys_s[slot] = k[q];
-      if constexpr (KV) vals_s[slot] = v[q];
+      if constexpr (KEEP_ID) id = __byte_perm(idk[c], 0u, 0x4440u + j);
+      else id = id_of(kk[j], q);
+      sl[j] = (FULL || b0 + q < nt) ? *reinterpret_cast<const uint16_t *>(cb + (id << 9)) : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int q = 4 * c + j;
+      if (FULL || b0 + q < nt) {
+        const uint32_t slot = sl[j] + __byte_perm(rk[c], 0u, 0x4440u + j);
+        keys_s[slot] = kk[j];
+        if constexpr (KV) vals_s[slot] = vv[j];
+      }
     }
   }
   fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA (async proxy)
@@ -258,6 +321,7 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
 
   // ---- 4. bucket runs: 8 threads per bucket -- 3 head keys, 3 tail keys,
   //         and the TMA bulk store(s) of the 16-byte-aligned body
+  if (p.dbg == 1) return;  // ablation: no stores
   {
     const uint32_t b = tid >> 3, sub = tid & 7;
     if (b < m) {
@@ -280,14 +344,14 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   }
 }
 
-template <int KIND, bool KV, int LOGMP, bool IDS8>
-__global__ void __launch_bounds__(kThreads, KV ? 2 : 3)
+template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT>
+__global__ void __launch_bounds__(kThreads, (KV || KPT > 16) ? 2 : 3)
 k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const void *__restrict__ ids, const uint32_t *__restrict__ G,
              uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
-             uint32_t L, const __grid_constant__ BucketParams p, int reverse) {
-  using Ly = K3pLayout<LOGMP, KV, IDS8>;
-  constexpr int T = Ly::T, STAGES = Ly::STAGES, CW = Ly::CW, MP = Ly::MP;
+             uint32_t L, const __grid_constant__ BucketParams p) {
+  using Ly = K3pLayout<LOGMP, KV, IDS8, KPT>;
+  constexpr int T = Ly::T, STAGES = Ly::STAGES, CW = Ly::CW, MP = Ly::MP, K = Ly::K;
   extern __shared__ __align__(128) uint32_t sm[];
   uint32_t *stk = sm + Ly::O_STK;
   uint32_t *stv = sm + Ly::O_STV;
@@ -309,7 +373,7 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   // prologue: STAGES tiles in flight
 #pragma unroll
   for (int s = 0; s < STAGES; ++s) {
-    if ((uint32_t)s < iters) k3p_prefetch<KV, IDS8, T>(stk, stv, sti, s, keys, vals, ids, tile_of(s), n, beta);
+    if ((uint32_t)s < iters) k3p_prefetch<KV, IDS8, T, K>(stk, stv, sti, s, keys, vals, ids, tile_of(s), n, beta);
     cp_async_commit();
   }
   uint32_t gnext = 0;
@@ -337,11 +401,11 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const int st = (int)(it % STAGES);
     uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
     begin_tile(it, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, true>(stk + st * T, stv + st * T, sti + st * (T / 4), ids, keys_out, vals_out,
-                                          tile * T, T, p, sm, beta, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, true>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
+                                               vals_out, tile * T, T, p, sm, beta, meta);
     // refill this stage with tile it + STAGES (own chunks only; already consumed)
     if (it + STAGES < iters)
-      k3p_prefetch<KV, IDS8, T>(stk, stv, sti, st, keys, vals, ids, tile_of(it + STAGES), n, beta);
+      k3p_prefetch<KV, IDS8, T, K>(stk, stv, sti, st, keys, vals, ids, tile_of(it + STAGES), n, beta);
     cp_async_commit();
   }
   if (has_tail) {
@@ -349,10 +413,50 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const int st = (int)(it % STAGES);
     uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
     begin_tile(it, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, false>(stk + st * T, stv + st * T, sti + st * (T / 4), ids, keys_out,
-                                           vals_out, tile * T, (uint32_t)(n - tile * T), p, sm, beta, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, false>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
+                                                vals_out, tile * T, (uint32_t)(n - tile * T), p, sm, beta, meta);
   }
   bulk_wait_read0();
+}
+
+// ------------------------------------------------------------------ host launcher
+template <typename Kern>
+inline cudaError_t k3p_launch_one(Kern k, size_t smem, const K3pArgs &a) {
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, smem);
+  if (per_sm <= 0) per_sm = 1;
+  const unsigned grid = (unsigned)umin64_host(a.L, (uint64_t)a.sms * per_sm);
+  k<<<grid, kThreads, smem, a.stream>>>(a.keys, a.vals, a.ids, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+  return cudaGetLastError();
+}
+
+template <int KIND, bool KV, int LOGMP, int KPT>
+inline cudaError_t k3p_launch_l(const K3pArgs &a) {
+  if constexpr (KIND == IDS) {
+    if (a.id_bytes == 1)
+      return k3p_launch_one(k3p_postscan<KIND, KV, LOGMP, true, KPT>, K3pLayout<LOGMP, KV, true, KPT>::BYTES, a);
+  }
+  return k3p_launch_one(k3p_postscan<KIND, KV, LOGMP, false, KPT>, K3pLayout<LOGMP, KV, false, KPT>::BYTES, a);
+}
+
+template <int KIND, bool KV, int KPT>
+inline cudaError_t k3p_launch_kv(const K3pArgs &a) {
+  uint32_t l = 1;
+  while ((1u << l) < a.m) ++l;
+  switch (l) {
+    case 1: return k3p_launch_l<KIND, KV, 1, KPT>(a);
+    case 2: return k3p_launch_l<KIND, KV, 2, KPT>(a);
+    case 3: return k3p_launch_l<KIND, KV, 3, KPT>(a);
+    case 4: return k3p_launch_l<KIND, KV, 4, KPT>(a);
+    default: return k3p_launch_l<KIND, KV, 5, KPT>(a);
+  }
+}
+
+template <int KIND>
+inline cudaError_t k3p_launch(const K3pArgs &a) {
+  if (a.kpt == 32) return a.vals ? k3p_launch_kv<KIND, true, 32>(a) : k3p_launch_kv<KIND, false, 32>(a);
+  return a.vals ? k3p_launch_kv<KIND, true, 16>(a) : k3p_launch_kv<KIND, false, 16>(a);
 }
 
 }  // namespace ms

@@ -1,0 +1,28 @@
+// ms_k3p_args.h -- host-side entry points of the persistent K3 (m <= 32), one TU per bucket kind.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "ms_device.cuh"
+
+namespace ms {
+
+struct K3pArgs {
+  const uint32_t *keys, *vals;
+  const void *ids;
+  const uint32_t *G;
+  uint32_t *keys_out, *vals_out;
+  uint32_t n, L, m, id_bytes, kpt;
+  const BucketParams *bp;  // host copy, passed by value to the kernel
+  int sms;
+  cudaStream_t stream;
+};
+
+cudaError_t k3p_launch_lowbits(const K3pArgs &a);
+cudaError_t k3p_launch_shiftc(const K3pArgs &a);
+cudaError_t k3p_launch_delta(const K3pArgs &a);
+cudaError_t k3p_launch_splitters(const K3pArgs &a);
+cudaError_t k3p_launch_ids(const K3pArgs &a);
+
+}  // namespace ms
