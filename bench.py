@@ -343,20 +343,102 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True):
     return res
 
 
+def bench_dist(name, cfg, K, Wm, device, world, rank, backend):
+    """N > 1: the sharded multisplit (dist.py): local ms_run + count all-gather + grouped
+    point-to-point exchange into balanced output windows.  Weak scaling: every rank holds
+    cfg['n'] keys (global indices rank*n ...).  Time = CUDA events around each whole
+    collective step on the launch stream, summed over K steps, max over ranks."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_ashkianidmo16_b200 as P
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import dist_multisplit
+    n = cfg["n"]
+    keys, vals = inputs_torch(cfg, n, rank * n, device)
+    spec = spec_of(cfg)
+    plan = P.Plan(spec, n, with_values=cfg["kv"])
+    ex_dev = "cpu" if backend == "gloo" else device   # gloo: stage the exchange through host memory
+
+    def local(k, v):
+        ko, vo, off = plan.run(k, v)
+        if ex_dev == "cpu":
+            return ko.cpu(), (vo.cpu() if vo is not None else None), off.cpu()
+        return ko, vo, off
+
+    flush_buf = torch.empty(512 << 20, dtype=torch.uint8, device=device)
+    for _ in range(Wm):
+        dist_multisplit(keys, vals, spec, local=local)
+    torch.cuda.synchronize()
+    dist.barrier()
+    s = torch.cuda.current_stream()
+    tot_ms = 0.0
+    clocks = ClockSampler(torch.cuda.current_device())
+    with clocks:
+        for _ in range(K):
+            flush_buf.fill_(1)
+            torch.cuda.synchronize()
+            dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            wk, wv, offg, ws = dist_multisplit(keys, vals, spec, local=local)
+            e1.record(s)
+            torch.cuda.synchronize()
+            tot_ms += e0.elapsed_time(e1)
+    dist.barrier()
+    tot_ms = max_over_ranks(tot_ms, world, device)
+    ms_step = tot_ms / K
+    value = n * world / (ms_step * 1e-3) / 1e9
+    # e2e: pinned host shard -> device, sharded multisplit, window -> pinned host
+    kh = keys.cpu().pin_memory()
+    vh = vals.cpu().pin_memory() if vals is not None else None
+    Ke = max(2, min(K, 5))
+    e2e_ms = 0.0
+    for _ in range(Ke):
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        kd = kh.to(device, non_blocking=True)
+        vd = vh.to(device, non_blocking=True) if vh is not None else None
+        wk, wv, offg, ws = dist_multisplit(kd, vd, spec, local=local)
+        wk_h = wk.to("cpu", non_blocking=True)
+        wv_h = wv.to("cpu", non_blocking=True) if wv is not None else None
+        e1.record(s)
+        torch.cuda.synchronize()
+        e2e_ms += e0.elapsed_time(e1)
+    e2e_ms = max_over_ranks(e2e_ms, world, device) / Ke
+    h2d = n * 4 * (2 if vals is not None else 1)
+    d2h = wk.numel() * 4 * (2 if vals is not None else 1)
+    del keys, vals, flush_buf
+    return {"value": value, "ms_per_step": ms_step, "clocks": clocks.result(),
+            "e2e": {"value": n * world / (e2e_ms * 1e-3) / 1e9, "unit": "G keys/s", "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms}}
+
+
 def run_ours(args, cfg, world, rank, local):
     import torch
-    device = torch.device("cuda", local)
+    # one process per GPU; ranks beyond the visible GPUs share them (only for the gloo test mode)
+    device = torch.device("cuda", local % max(1, torch.cuda.device_count()))
     torch.cuda.set_device(device)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=device)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=device)
+        else:
+            dist.init_process_group(args.dist_backend)
     from paper_conf_ppopp_ashkianidmo16_b200 import build as b
     if rank == 0:
         b.build()
     barrier(world)
-    res = bench_config(args.config, cfg, args.steps, args.warmup, device, world, rank)
+    # the per-rank kernels, traced (roofline, stages); at N = 1 this IS the headline step
+    res = bench_config(args.config, cfg, args.steps, args.warmup, device, world, rank, with_e2e=(world == 1))
+    if world > 1:
+        d = bench_dist(args.config, cfg, args.steps, args.warmup, device, world, rank, args.dist_backend)
+        local_value = res["value"]
+        res.update(value=d["value"], ms_per_step=d["ms_per_step"], clocks=d["clocks"], e2e=d["e2e"])
+        res["local_step"] = {"value_if_independent": round(local_value, 3),
+                             "note": "same kernels without the exchange (independent shards), max over ranks"}
     extra = {}
-    if not args.no_extra:
+    if not args.no_extra and world == 1:
         for nm in args.extra.split(","):
             if nm and nm in CONFIGS and nm != args.config:
                 r = bench_config(nm, CONFIGS[nm], max(5, args.steps // 4), 3, device, world, rank, with_e2e=False)
@@ -382,13 +464,17 @@ def run_ours(args, cfg, world, rank, local):
             "config": {"workload": args.config, "desc": cfg["desc"], "n_per_gpu": cfg["n"], "m": cfg["m"],
                        "kind": cfg["kind"], "kv": cfg["kv"], "dist": cfg["dist"],
                        "l2": "flushed between timed steps (512 MiB write, outside the timed kernels)",
-                       "parallelism": f"independent shards x{world}" if world > 1 else "single GPU"},
+                       "parallelism": (f"sharded multisplit x{world}: local ms_run + NCCL count all-gather + "
+                                       f"grouped send/recv into balanced windows ({args.dist_backend})")
+                       if world > 1 else "single GPU"},
             "roofline": res["roofline"], "e2e": res["e2e"], "cpu_baseline": cpu,
             "gpu_launches": res["gpu_launches"], "clocks": res["clocks"],
             "stages_ms": res["stages_ms"], "whole_step_frac": round(res["whole_step_frac"], 4),
             "whole_step_hbm_gbs": round(res["whole_step_hbm_gbs"], 1),
             "tile": res["tile"], "variant": res["variant"], "extra": extra,
         }
+        if "local_step" in res:
+            out["local_step"] = res["local_step"]
         print(json.dumps(out), flush=True)
     if world > 1:
         import torch.distributed as dist
@@ -405,6 +491,8 @@ def main():
     ap.add_argument("--extra", default="NSko,NSkv,C4ko,C3")
     ap.add_argument("--no-extra", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="N>1 exchange backend (gloo: host-staged, for testing on one GPU)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -159,6 +159,42 @@ ms_status ms_plan_trace(ms_plan_t plan, int enable);
 ms_status ms_plan_trace_read(ms_plan_t plan, float *stage_ms, int32_t max_runs, int32_t *runs,
                              int32_t *stages);
 
+/* ---------------------------------------------------------------------------
+ * Sharded multisplit over P ranks: Eq. (2) with the
+ * GPUs as the outermost subproblem level.  Rank g multisplits its shard locally
+ * (ms_run), the m-vectors of per-rank bucket counts h[g][b] are all-gathered,
+ * and every element of rank g's local bucket b at local position i goes to
+ * global position B[b] + sum_{g'<g} h[g'][b] + (i - off_g[b]), where
+ * B[b] = sum_{b'<b} sum_g h[g][b'].  The global output is cut into P balanced
+ * windows (rank r owns [r*q + min(r, rem), ...), q = N/P, rem = N%P), so the
+ * concatenation of the windows is the single-GPU stable multisplit of the
+ * concatenated shards.  Because rank g's local output is monotone in global
+ * position, it leaves in at most m+P-1 contiguous pieces.
+ *
+ * ms_dist_pieces (HOST function, no device access): from the all-gathered
+ * counts (host, P*m u64, row g = rank g), compute for rank `rank`:
+ *   send[k] = {src_off (local output offset), len, peer (dst rank), dst_off (offset in the peer's window)}
+ *   recv[k] = {src_off (offset in the sender's local output), len, peer (src rank), dst_off (offset in my window)}
+ * in the order both sides must issue them (buckets ascending per peer), plus
+ * the global bucket starts offsets_global[m+1] (u64) and this rank's window
+ * [*win_start, *win_start + *win_len).  The arrays hold at most m+P-1 (send)
+ * and m*P (recv) entries; *n_send / *n_recv report the counts.  Pieces with
+ * peer == rank are local copies.  Returns MS_ERR_INVALID_ARG on bad sizes or if
+ * a capacity is too small.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+  uint64_t src_off;
+  uint64_t len;
+  int32_t peer;
+  int32_t pad_;
+  uint64_t dst_off;
+} ms_piece;
+
+ms_status ms_dist_pieces(int32_t nranks, int32_t rank, uint32_t m, const uint64_t *counts,
+                         ms_piece *send, int32_t send_cap, int32_t *n_send, ms_piece *recv,
+                         int32_t recv_cap, int32_t *n_recv, uint64_t *offsets_global,
+                         uint64_t *win_start, uint64_t *win_len);
+
 #ifdef __cplusplus
 }
 #endif

@@ -29,7 +29,7 @@ EXPORTS = [
     "ms_plan_create", "ms_plan_workspace_size", "ms_plan_geometry", "ms_run",
     "ms_plan_workspace_size_host", "ms_run_host", "ms_prescan", "ms_scan", "ms_postscan",
     "ms_bucket_ids", "ms_plan_check", "ms_plan_destroy", "ms_status_string",
-    "ms_plan_last_launches", "ms_plan_trace", "ms_plan_trace_read",
+    "ms_plan_last_launches", "ms_plan_trace", "ms_plan_trace_read", "ms_dist_pieces",
 ]
 
 
@@ -79,6 +79,8 @@ def lib():
     L.ms_plan_last_launches.argtypes = [P]
     L.ms_plan_trace.argtypes = [P, ctypes.c_int]
     L.ms_plan_trace_read.argtypes = [P, P, I32, ctypes.POINTER(I32), ctypes.POINTER(I32)]
+    L.ms_dist_pieces.argtypes = [I32, I32, U32, P, P, I32, ctypes.POINTER(I32), P, I32, ctypes.POINTER(I32), P,
+                                 ctypes.POINTER(U64), ctypes.POINTER(U64)]
     for name in EXPORTS:
         f = getattr(L, name)
         if name != "ms_status_string":

@@ -1,0 +1,143 @@
+"""Sharded multisplit: host planning + the exchange, on CPU with gloo (world size 2..4).
+
+The local per-rank step here is the CPU oracle (test infrastructure) so the
+whole N>1 orchestration -- count all-gather, ms_dist_pieces planning (native,
+libms.so), grouped point-to-point exchange -- runs without a GPU; the product
+path uses ms_run on the GPU for the local step.  Expected: the concatenation of
+the rank windows equals the single-GPU stable multisplit of the concatenated
+shards."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import workloads as W
+from paper_conf_ppopp_ashkianidmo16_b200.dist import dist_multisplit, dist_pieces
+from paper_conf_ppopp_ashkianidmo16_b200.api import BucketSpec
+
+
+# ------------------------------------------------------------ planning alone
+@pytest.mark.parametrize("P,m", [(1, 1), (2, 3), (3, 32), (4, 8), (8, 32), (8, 256), (5, 1)])
+def test_pieces_cover_and_match(P, m):
+    rng = np.random.default_rng(P * 100 + m)
+    for trial in range(20):
+        counts = rng.integers(0, 50, size=(P, m)).astype(np.uint64)
+        if trial % 4 == 0:
+            counts[:, m // 2] *= 20            # skew: one heavy bucket
+        if trial % 5 == 0:
+            counts[rng.integers(P)] = 0         # an empty shard
+        N = int(counts.sum())
+        plans = [dist_pieces(P, r, m, counts) for r in range(P)]
+        B = np.concatenate([[0], np.cumsum(counts.sum(axis=0))]).astype(np.uint64)
+        for r in range(P):
+            assert np.array_equal(plans[r][2], B)                    # global bucket starts
+        wins = [(p[3], p[4]) for p in plans]
+        assert wins[0][0] == 0 and sum(w[1] for w in wins) == N
+        assert max(w[1] for w in wins) - min(w[1] for w in wins) <= 1  # balanced windows
+        for r in range(P - 1):
+            assert wins[r][0] + wins[r][1] == wins[r + 1][0]
+        cover = np.zeros(N, dtype=np.int64)
+        for g in range(P):
+            send = plans[g][0]
+            assert len(send) <= m + P - 1                            # monotone output: <= m+P-1 pieces
+            assert sum(p[1] for p in send) == int(counts[g].sum())   # every local element leaves once
+            for s_off, ln, peer, d_off in send:
+                cover[wins[peer][0] + d_off: wins[peer][0] + d_off + ln] += 1
+                # the matching receive exists at the peer with the same geometry
+                assert (s_off, ln, g, d_off) in plans[peer][1]
+        assert np.all(cover == 1)
+        for r in range(P):                                           # receives tile the window exactly
+            assert sum(p[1] for p in plans[r][1]) == wins[r][1]
+
+
+def test_pieces_follow_eq2():
+    """Global position of local element i of bucket b on rank g = B[b] + sum_{g'<g} h[g'][b] + (i - off_g[b])."""
+    P, m = 3, 4
+    counts = np.array([[2, 0, 3, 1], [1, 1, 0, 4], [0, 2, 2, 0]], dtype=np.uint64)
+    B = np.concatenate([[0], np.cumsum(counts.sum(axis=0))])
+    for g in range(P):
+        send, _, _, _, _ = dist_pieces(P, g, m, counts)
+        off = np.concatenate([[0], np.cumsum(counts[g])])
+        gpos = {}
+        plans = [dist_pieces(P, r, m, counts) for r in range(P)]
+        for s_off, ln, peer, d_off in send:
+            for k in range(ln):
+                gpos[s_off + k] = plans[peer][3] + d_off + k
+        for b in range(m):
+            for i in range(int(off[b]), int(off[b + 1])):
+                assert gpos[i] == B[b] + counts[:g, b].sum() + (i - off[b])
+
+
+# ------------------------------------------------------------ full exchange with gloo
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _shard_sizes(P, n, mode):
+    if mode == "equal":
+        return [n // P + (1 if r < n % P else 0) for r in range(P)]
+    sizes = [(n * (r + 1)) // (P * (P + 1) // 2) for r in range(P)]   # unequal, rank-increasing
+    sizes[-1] += n - sum(sizes)
+    if mode == "empty":
+        sizes[0], sizes[-1] = 0, sizes[-1] + sizes[0]
+    return sizes
+
+
+def _case(kind, m):
+    if kind == "splitters":
+        spl = W.gen_splitters(m, 3)
+        return BucketSpec.from_splitters(spl.tolist()), oracle.Spec("splitters", m, splitters=spl), W.ranges_splitters(spl)
+    delta = max(1, (1 << 32) // m)
+    return BucketSpec.delta_range(m, delta), oracle.Spec("delta", m, delta=delta), W.ranges_delta(m, delta)
+
+
+def _worker(rank, P, port, n, kind, m, dist_name, mode, kv):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=P)
+    try:
+        spec, ospec, ranges = _case(kind, m)
+        sizes = _shard_sizes(P, n, mode)
+        start = sum(sizes[:rank])
+        keys = W.keys_np(sizes[rank], 11, dist_name, m, ranges, start=start) if dist_name != "uniform" else \
+            W.keys_np(sizes[rank], 11, start=start)
+        vals = W.values_np(sizes[rank], 11, "index", start=start) if kv else None
+
+        def local(k, v):  # CPU oracle as the local step (test infrastructure)
+            ko, vo, off = oracle.multisplit(ospec, k.numpy().view(np.uint32),
+                                            None if v is None else v.numpy().view(np.uint32))
+            t = lambda a: torch.from_numpy(a.view(np.int32).copy())  # noqa: E731
+            return t(ko), (t(vo) if vo is not None else None), torch.from_numpy(off.astype(np.int64))
+
+        kt = torch.from_numpy(keys.view(np.int32).copy())
+        vt = torch.from_numpy(vals.view(np.int32).copy()) if kv else None
+        wk, wv, offg, ws = dist_multisplit(kt, vt, spec, local=local)
+        # expected: oracle of the concatenated input, sliced to my window
+        allk = W.keys_np(n, 11, dist_name, m, ranges) if dist_name != "uniform" else W.keys_np(n, 11)
+        allv = W.values_np(n, 11, "index") if kv else None
+        eko, evo, eoff = oracle.multisplit(ospec, allk, allv)
+        assert np.array_equal(offg, eoff)
+        assert np.array_equal(wk.numpy().view(np.uint32), eko[ws:ws + wk.numel()])
+        if kv:
+            assert np.array_equal(wv.numpy().view(np.uint32), evo[ws:ws + wv.numel()])
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("P,kind,m,dist_name,mode,kv", [
+    (2, "delta", 8, "uniform", "equal", True),
+    (3, "splitters", 32, "hot", "unequal", True),
+    (4, "delta", 256, "binomial", "empty", False),
+    (4, "splitters", 5, "one", "equal", True),
+])
+def test_dist_multisplit_gloo(P, kind, m, dist_name, mode, kv):
+    n = 20011
+    mp.spawn(_worker, args=(P, _free_port(), n, kind, m, dist_name, mode, kv), nprocs=P, join=True)
