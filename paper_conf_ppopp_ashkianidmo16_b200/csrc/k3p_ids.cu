@@ -1,6 +1,9 @@
-// k3p_ids.cu -- instantiates the persistent K3 (ms_k3_blocked.cuh) for whatBucket kind IDS.
+// k3p_ids.cu -- instantiates the K3 variants for whatBucket kind IDS:
+// persistent blocked-rank K3 (m <= 32, ms_k3_blocked.cuh) and warp-ballot K3 (m > 32, ms_k3_warp.cuh).
 #include "ms_k3_blocked.cuh"
+#include "ms_k3_warp.cuh"
 
 namespace ms {
 cudaError_t k3p_launch_ids(const K3pArgs &a) { return k3p_launch<IDS>(a); }
+cudaError_t k3w_launch_ids(const K3pArgs &a) { return k3w_launch<IDS>(a); }
 }  // namespace ms

@@ -1,6 +1,9 @@
-// k3p_shiftc.cu -- instantiates the persistent K3 (ms_k3_blocked.cuh) for whatBucket kind SHIFTC.
+// k3p_shiftc.cu -- instantiates the K3 variants for whatBucket kind SHIFTC:
+// persistent blocked-rank K3 (m <= 32, ms_k3_blocked.cuh) and warp-ballot K3 (m > 32, ms_k3_warp.cuh).
 #include "ms_k3_blocked.cuh"
+#include "ms_k3_warp.cuh"
 
 namespace ms {
 cudaError_t k3p_launch_shiftc(const K3pArgs &a) { return k3p_launch<SHIFTC>(a); }
+cudaError_t k3w_launch_shiftc(const K3pArgs &a) { return k3w_launch<SHIFTC>(a); }
 }  // namespace ms

@@ -114,10 +114,6 @@ void set_smem(K kernel, size_t bytes) {
 
 size_t k1_smem(uint32_t m) { return kMaxM * 4 + (size_t)m * kThreads; }
 
-size_t k3_smem(int R, bool kv, bool id8) {
-  size_t T = 256u * R;
-  return T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
-}
 
 // ---------------------------------------------------------------- dispatch
 template <int KIND>
@@ -138,27 +134,6 @@ cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *key
     default: MS_K1(32) break;
   }
 #undef MS_K1
-  return cudaGetLastError();
-}
-
-template <int KIND, bool KV>
-cudaError_t launch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
-                      const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
-                      uint32_t *vo, uint32_t n, cudaStream_t s) {
-  constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC);
-#define MS_K3(R)                                                                             \
-  {                                                                                          \
-    auto k = k3_postscan<KIND, KV, R>;                                                       \
-    size_t smem = k3_smem(R, KV, id8);                                                       \
-    set_smem(k, smem);                                                                       \
-    k<<<(unsigned)g.L, kThreads, smem, s>>>(keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->bp); \
-  }
-  switch (g.R) {
-    case 8: MS_K3(8) break;
-    case 16: MS_K3(16) break;
-    default: MS_K3(32) break;
-  }
-#undef MS_K3
   return cudaGetLastError();
 }
 
@@ -188,10 +163,9 @@ int sm_count() {
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                         uint32_t *vo, uint32_t n, cudaStream_t s) {
-  const bool kv = vals != nullptr;
+  K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
+            p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, &p->bp, sm_count(), s};
   if (p->spec.m <= 32) {  // persistent blocked-rank K3 (ms_k3_blocked.cuh), one TU per kind
-    K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes, p->kpt, &p->bp,
-              sm_count(), s};
     switch (p->kkind) {
       case LOWBITS: return k3p_launch_lowbits(a);
       case SHIFTC: return k3p_launch_shiftc(a);
@@ -200,17 +174,13 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
       default: return k3p_launch_ids(a);
     }
   }
-#define MS_K3K(KIND)                                                     \
-  return kv ? launch_k3<KIND, true>(p, g, keys, vals, ids, G, ko, vo, n, s) \
-            : launch_k3<KIND, false>(p, g, keys, vals, ids, G, ko, vo, n, s);
-  switch (p->kkind) {
-    case LOWBITS: MS_K3K(LOWBITS)
-    case SHIFTC: MS_K3K(SHIFTC)
-    case DELTA: MS_K3K(DELTA)
-    case SPLITTERS: MS_K3K(SPLITTERS)
-    default: MS_K3K(IDS)
+  switch (p->kkind) {  // m > 32: warp-ballot K3 (ms_k3_warp.cuh)
+    case LOWBITS: return k3w_launch_lowbits(a);
+    case SHIFTC: return k3w_launch_shiftc(a);
+    case DELTA: return k3w_launch_delta(a);
+    case SPLITTERS: return k3w_launch_splitters(a);
+    default: return k3w_launch_ids(a);
   }
-#undef MS_K3K
 }
 
 ms_status check_ws(const ms_plan_s *p, uint64_t n, void *ws, size_t ws_bytes, Geometry *g) {

@@ -1,0 +1,221 @@
+// ms_k3_warp.cuh -- K3 post-scan for m > 32: warp-striped rounds, Alg. 3 ballot ranks (sm_100a).
+#pragma once
+#include "ms_k3p_args.h"
+
+namespace ms {
+
+// ============================================================== K3 post-scan
+// Recompute ids (footnote 6), stable tile-local ranks, a local
+// stable multisplit of the tile in shared memory (§4 "reordering",
+// P:689-713; §5.2.2 block-level reordering P:1262-1301) and coalesced stores
+// of each bucket run to G[j][tile] + (slot - S_t[j]).
+//
+// Tile = 8 warps x R rounds x 32 keys; warp w owns the contiguous segment
+// [w*32R, (w+1)*32R) and walks it in rounds of 32 consecutive keys, so
+// (warp, round, lane) order IS input order and ranks are stable.
+// Per round the LOGM ballots of Alg. 3 (one ballot per id bit,
+// compile-time LOGM) give each lane the mask of same-bucket lanes (on sm_100
+// __match_any_sync is ~2x dearer than 8 ballots when lanes hold distinct ids:
+// it runs on the ADU pipe), popc(mask & lanemask_lt) is the
+// exclusive rank (reading #4), and the highest lane of each group advances
+// the warp's shared-memory counter for that bucket.  Cross-warp exclusive prefixes +
+// the tile's bucket starts S_t then give each key its shared-memory slot
+// (Eq. (2) one level down).  Keys (and values) arrive by one TMA
+// bulk copy per array (UBLKCP) on an mbarrier.
+template <int KIND, bool KV, int R, int LOGM, bool FULL>
+__device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
+                                        uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
+                                        uint64_t base, uint32_t nt, const BucketParams &p,
+                                        uint32_t *keys_s, uint32_t *vals_s, uint32_t *cnt_s,
+                                        uint32_t *gD_s, const uint32_t *spl_s, uint8_t *id8_s,
+                                        uint32_t *wsum, uint32_t gcol) {
+  constexpr int SEG = 32 * R;
+  constexpr bool ID8 = (KIND != LOWBITS && KIND != SHIFTC);
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t m = p.m;
+  const uint32_t lt = lanemask_lt(), gt = lanemask_gt();
+  uint32_t *cnt_w = cnt_s + warp * kMaxM;
+  const uint32_t seg0 = warp * SEG + lane;
+
+  uint32_t idr[KIND == IDS ? R : 1];
+  if constexpr (KIND == IDS) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint32_t pos = seg0 + r * 32;
+      idr[r] = (FULL || pos < nt) ? load_id(ids, base + pos, p) : 0xFFFFFFFFu;
+    }
+  }
+
+  // ---- phase 1: stable ranks within the warp's segment
+  uint32_t kreg[R];
+  uint32_t vreg[KV ? R : 1];
+  uint32_t pk[R];  // (rank within warp segment) << 8 | id
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t pos = seg0 + r * 32;
+    const bool valid = FULL || pos < nt;
+    const uint32_t key = keys_s[pos];
+    uint32_t id;
+    if constexpr (KIND == IDS) id = idr[r];
+    else id = valid ? bucket_of_key<KIND>(key, p, spl_s) : 0xFFFFFFFFu;
+    uint32_t peers = FULL ? 0xFFFFFFFFu : __ballot_sync(0xFFFFFFFFu, valid);
+#pragma unroll
+    for (int b = 0; b < LOGM; ++b) {
+      const uint32_t bit = (id >> b) & 1u;
+      const uint32_t vote = __ballot_sync(0xFFFFFFFFu, bit);
+      peers &= bit ? vote : ~vote;
+    }
+    const uint32_t rank = __popc(peers & lt);
+    uint32_t before = 0;
+    if (valid) before = cnt_w[id];
+    __syncwarp();
+    if (valid && (peers & gt) == 0) cnt_w[id] = before + __popc(peers);
+    __syncwarp();
+    kreg[r] = key;
+    if constexpr (KV) vreg[r] = vals_s[pos];
+    pk[r] = ((before + rank) << 8) | (id & 255u);
+  }
+  __syncthreads();
+
+  // ---- per-bucket cross-warp exclusive prefix, tile bucket starts S_t
+  uint32_t tot = 0;
+  if (tid < m) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) {
+      const uint32_t c = cnt_s[w * kMaxM + tid];
+      cnt_s[w * kMaxM + tid] = tot;
+      tot += c;
+    }
+  }
+  const uint32_t incl = warp_incl_scan(tot, lane);
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  uint32_t wpre = 0;
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) wpre += (w < (int)warp) ? wsum[w] : 0u;
+  const uint32_t S = wpre + incl - tot;  // exclusive scan of the tile histogram
+  if (tid < m) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] += S;
+    gD_s[tid] = gcol - S;
+  }
+  __syncthreads();
+
+  // ---- local multisplit of the tile into shared memory (in place)
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (FULL || seg0 + r * 32 < nt) {
+      const uint32_t id = pk[r] & 255u;
+      const uint32_t slot = cnt_w[id] + (pk[r] >> 8);
+      keys_s[slot] = kreg[r];
+      if constexpr (KV) vals_s[slot] = vreg[r];
+      if constexpr (ID8) id8_s[slot] = (uint8_t)id;
+    }
+  }
+  __syncthreads();
+
+  // ---- coalesced stores of the bucket runs
+  auto store = [&](uint32_t i) {
+    const uint32_t k = keys_s[i];
+    uint32_t id;
+    if constexpr (ID8) id = id8_s[i];
+    else id = bucket_of_key<KIND>(k, p, spl_s);
+    const uint32_t dst = gD_s[id] + i;
+    __stcs(keys_out + dst, k);
+    if constexpr (KV) __stcs(vals_out + dst, vals_s[i]);
+  };
+  if constexpr (FULL) {
+#pragma unroll 4
+    for (int j = 0; j < R; ++j) store(j * kThreads + tid);
+  } else {
+    for (uint32_t i = tid; i < nt; i += kThreads) store(i);
+  }
+}
+
+template <int KIND, bool KV, int R, int LOGM>
+__global__ void __launch_bounds__(kThreads)
+k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
+            const void *__restrict__ ids, const uint32_t *__restrict__ G,
+            uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
+            uint32_t L, const __grid_constant__ BucketParams p) {
+  constexpr int T = kThreads * R;
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  uint32_t *keys_s = reinterpret_cast<uint32_t *>(smem_raw);
+  uint32_t *vals_s = keys_s + T;
+  uint32_t *cnt_s = vals_s + (KV ? T : 0);     // [8][256] per-warp counters
+  uint32_t *gD_s = cnt_s + kWarps * kMaxM;     // [256] G[j][tile] - S_t[j]
+  uint32_t *spl_s = gD_s + kMaxM;              // [256] padded splitters
+  uint8_t *id8_s = reinterpret_cast<uint8_t *>(spl_s + kMaxM);  // [T]
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ uint32_t wsum[kWarps];
+
+  const uint32_t tid = threadIdx.x;
+  const uint32_t tile = blockIdx.x;
+  const uint64_t base = (uint64_t)tile * T;
+  const uint32_t nt = (uint32_t)umin64(T, n - base);
+  const bool full = (nt == T);
+  const uint32_t m = p.m;
+
+  if (full) {
+    if (tid == 0) {
+      mbar_init(&bar, 1);
+      fence_mbar_init();
+      mbar_arrive_expect_tx(&bar, (KV ? 2u : 1u) * T * 4u);
+      bulk_g2s(keys_s, keys + base, T * 4u, &bar);
+      if constexpr (KV) bulk_g2s(vals_s, vals + base, T * 4u, &bar);
+    }
+  } else {
+    for (uint32_t i = tid; i < nt; i += kThreads) {
+      keys_s[i] = keys[base + i];
+      if constexpr (KV) vals_s[i] = vals[base + i];
+    }
+  }
+  // per-bucket setup while the copy is in flight
+  uint32_t gcol = 0;
+  if (tid < m) gcol = __ldg(G + (uint64_t)tid * L + tile);
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] = 0;  // kThreads == kMaxM
+  if constexpr (KIND == SPLITTERS) {
+    if (tid < (1u << p.logm)) spl_s[tid] = p.spl[tid];
+  }
+  __syncthreads();
+  if (full) {
+    mbar_wait(&bar, 0);
+    k3_tile<KIND, KV, R, LOGM, true>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+                               spl_s, id8_s, wsum, gcol);
+  } else {
+    k3_tile<KIND, KV, R, LOGM, false>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+                                spl_s, id8_s, wsum, gcol);
+  }
+}
+
+// ------------------------------------------------------------------ host launcher (m > 32)
+inline size_t k3w_smem(int R, bool kv, bool id8) {
+  const size_t T = 256u * R;
+  return T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
+}
+
+template <int KIND, bool KV, int R, int LOGM>
+inline cudaError_t k3w_launch_l(const K3pArgs &a) {
+  constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC);
+  auto k = k3_postscan<KIND, KV, R, LOGM>;
+  const size_t smem = k3w_smem(R, KV, id8);
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<a.L, kThreads, smem, a.stream>>>(a.keys, a.vals, a.ids, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+  return cudaGetLastError();
+}
+
+template <int KIND, bool KV, int R>
+inline cudaError_t k3w_launch_r(const K3pArgs &a) {
+  if (a.m <= 64) return k3w_launch_l<KIND, KV, R, 6>(a);
+  if (a.m <= 128) return k3w_launch_l<KIND, KV, R, 7>(a);
+  return k3w_launch_l<KIND, KV, R, 8>(a);
+}
+
+template <int KIND>
+inline cudaError_t k3w_launch(const K3pArgs &a) {
+  if (a.kpt == 8) return a.vals ? k3w_launch_r<KIND, true, 8>(a) : k3w_launch_r<KIND, false, 8>(a);
+  return a.vals ? k3w_launch_r<KIND, true, 16>(a) : k3w_launch_r<KIND, false, 16>(a);
+}
+
+}  // namespace ms

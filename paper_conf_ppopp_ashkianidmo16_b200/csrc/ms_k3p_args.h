@@ -24,5 +24,11 @@ cudaError_t k3p_launch_shiftc(const K3pArgs &a);
 cudaError_t k3p_launch_delta(const K3pArgs &a);
 cudaError_t k3p_launch_splitters(const K3pArgs &a);
 cudaError_t k3p_launch_ids(const K3pArgs &a);
+// m > 32: warp-ballot K3 (ms_k3_warp.cuh); kpt carries the rounds per warp R (8 or 16)
+cudaError_t k3w_launch_lowbits(const K3pArgs &a);
+cudaError_t k3w_launch_shiftc(const K3pArgs &a);
+cudaError_t k3w_launch_delta(const K3pArgs &a);
+cudaError_t k3w_launch_splitters(const K3pArgs &a);
+cudaError_t k3w_launch_ids(const K3pArgs &a);
 
 }  // namespace ms
