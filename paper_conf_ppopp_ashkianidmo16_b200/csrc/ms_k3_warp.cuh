@@ -58,13 +58,17 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
     uint32_t id;
     if constexpr (KIND == IDS) id = idr[r];
     else id = valid ? bucket_of_key<KIND>(key, p, spl_s) : 0xFFFFFFFFu;
-    uint32_t peers = FULL ? 0xFFFFFFFFu : __ballot_sync(0xFFFFFFFFu, valid);
+    // lanes whose id differs from mine in bit b = vote_b XOR sext(my bit b);
+    // one shifted copy of the id feeds both the vote predicate (its sign) and
+    // the sign-extension, and one LOP3 accumulates the difference mask
+    uint32_t diff = FULL ? 0u : ~__ballot_sync(0xFFFFFFFFu, valid);
 #pragma unroll
     for (int b = 0; b < LOGM; ++b) {
-      const uint32_t bit = (id >> b) & 1u;
-      const uint32_t vote = __ballot_sync(0xFFFFFFFFu, bit);
-      peers &= bit ? vote : ~vote;
+      const int32_t sh = (int32_t)(id << (31 - b));
+      const uint32_t vote = __ballot_sync(0xFFFFFFFFu, sh < 0);
+      diff |= vote ^ (uint32_t)(sh >> 31);
     }
+    const uint32_t peers = ~diff;
     const uint32_t rank = __popc(peers & lt);
     uint32_t before = 0;
     if (valid) before = cnt_w[id];
