@@ -277,9 +277,10 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->bp = bp;
   p->kkind = kkind;
   p->last_launches = 0;
-  // ablation override: MS_K3_KPT=16|32 keys per thread in K3 (m <= 32)
-  if (const char *e = getenv("MS_K3_KPT")) p->kpt = atoi(e) == 32 ? 32u : 16u;
+  // ablation overrides: MS_DEBUG_K3=1 drops K3's global stores;
+  // MS_K3_REVERSE=1 walks K3's tiles last-to-first
   if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
+  if (const char *e = getenv("MS_K3_REVERSE")) p->bp.reverse = atoi(e) ? 1u : 0u;
   *plan = p;
   return MS_OK;
 }

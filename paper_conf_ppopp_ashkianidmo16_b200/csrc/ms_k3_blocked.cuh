@@ -362,9 +362,18 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   // tiles blockIdx.x, blockIdx.x + gridDim.x, ...; the partial tile (if any)
   // is the last one overall, hence the last of its CTA: it is peeled off
   // the loop so its predicated code does not raise the loop's registers.
-  auto tile_of = [&](uint32_t it) -> uint64_t { return (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x; };
+  // p.reverse: walk tiles last-to-first, so the first tiles K3 reads are the
+  // ones K1 read last (still in the 126 MB L2); the partial tile is then the
+  // FIRST tile of CTA 0 instead of the last of its CTA.
+  const bool rev = p.reverse != 0;
+  auto tile_of = [&](uint32_t it) -> uint64_t {
+    const uint64_t t = (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x;
+    return rev ? (uint64_t)L - 1 - t : t;
+  };
   const uint32_t iters = blockIdx.x < L ? (L - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-  const bool has_tail = iters && (uint64_t)n < (uint64_t)L * T && tile_of(iters - 1) == L - 1;
+  const bool partial = (uint64_t)n < (uint64_t)L * T;
+  const bool tail_first = partial && rev && iters && blockIdx.x == 0;
+  const bool has_tail = partial && !rev && iters && tile_of(iters - 1) == L - 1;
   const uint32_t iters_full = iters - (has_tail ? 1 : 0);
 
   if constexpr (KIND == SPLITTERS) {
@@ -396,6 +405,16 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   };
 
   uint32_t it = 0;
+  if (tail_first) {
+    const uint64_t tile = tile_of(0);
+    uint32_t *meta = sm + Ly::O_META;
+    begin_tile(0, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, false>(stk, stv, sti, ids, keys_out, vals_out, tile * T,
+                                                (uint32_t)(n - tile * T), p, sm, beta, meta);
+    if (STAGES < iters) k3p_prefetch<KV, IDS8, T, K>(stk, stv, sti, 0, keys, vals, ids, tile_of(STAGES), n, beta);
+    cp_async_commit();
+    it = 1;
+  }
   for (; it < iters_full; ++it) {
     const uint64_t tile = tile_of(it);
     const int st = (int)(it % STAGES);
@@ -455,7 +474,6 @@ inline cudaError_t k3p_launch_kv(const K3pArgs &a) {
 
 template <int KIND>
 inline cudaError_t k3p_launch(const K3pArgs &a) {
-  if (a.kpt == 32) return a.vals ? k3p_launch_kv<KIND, true, 32>(a) : k3p_launch_kv<KIND, false, 32>(a);
   return a.vals ? k3p_launch_kv<KIND, true, 16>(a) : k3p_launch_kv<KIND, false, 16>(a);
 }
 

@@ -154,7 +154,7 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   __shared__ uint32_t wsum[kWarps];
 
   const uint32_t tid = threadIdx.x;
-  const uint32_t tile = blockIdx.x;
+  const uint32_t tile = p.reverse ? L - 1 - blockIdx.x : blockIdx.x;  // reverse: L2 reuse of K1's tail
   const uint64_t base = (uint64_t)tile * T;
   const uint32_t nt = (uint32_t)umin64(T, n - base);
   const bool full = (nt == T);

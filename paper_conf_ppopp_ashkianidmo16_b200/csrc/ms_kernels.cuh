@@ -47,7 +47,7 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   if (full) {
     const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
 #pragma unroll
-    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldcs(k4 + j * kThreads + tid);
+    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * kThreads + tid);  // cached: K3 reuses the tail from L2
   }
   // K2's look-back status words are cleared here (K1 precedes K2 in the stream).
   for (uint32_t i = tile * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;

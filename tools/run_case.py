@@ -16,9 +16,9 @@ keys, vals = bench.inputs_torch(cfg, cfg["n"], 0, "cuda")
 plan = P.Plan(bench.spec_of(cfg), cfg["n"], with_values=cfg["kv"], variant=variant)
 ko = torch.empty_like(keys)
 vo = torch.empty_like(vals) if vals is not None else None
-flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+flush = bench.L2Flush("cuda")
 for _ in range(reps):
-    flush.fill_(1)
+    flush()
     plan.run(keys, vals, keys_out=ko, vals_out=vo)
 torch.cuda.synchronize()
 print("ok", name, plan.geometry(cfg["n"]))
