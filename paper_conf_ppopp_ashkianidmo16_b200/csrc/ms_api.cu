@@ -26,7 +26,8 @@ struct ms_plan_s {
   uint32_t flags;
   BucketParams bp;
   int kkind;  // kernel-level Kind (ms_device.cuh)
-  uint32_t kpt = 16;  // K3 (m <= 32): keys per thread, tile T = 256 * kpt
+  uint32_t kpt = 16;  // K3 (m <= 32): keys per thread
+  uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt (MS_K3_NT)
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
   int tracing = 0;
@@ -86,7 +87,7 @@ struct Geometry {
 
 Geometry geometry(const ms_plan_s *p, uint64_t n) {
   Geometry g{};
-  g.R = rounds_for(p->spec.m, n, p->kpt);
+  g.R = rounds_for(p->spec.m, n, p->kpt * p->k3nt / 256);
   g.T = 256u * g.R;
   g.L = (n + g.T - 1) / g.T;
   g.hg_words = (uint64_t)p->spec.m * g.L;
@@ -121,17 +122,17 @@ cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *key
                       uint32_t n, uint32_t *H, uint64_t *zero_ptr, uint32_t zero_words,
                       uint32_t *flag, cudaStream_t s) {
   size_t smem = k1_smem(p->spec.m);
-#define MS_K1(KPT)                                                                         \
-  {                                                                                        \
-    auto k = k1_prescan<KIND, KPT>;                                                        \
-    set_smem(k, smem);                                                                     \
-    k<<<(unsigned)g.L, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, \
-                                            zero_words, flag);                             \
+#define MS_K1(KPT, SUBT)                                                                    \
+  {                                                                                          \
+    auto k = k1_prescan<KIND, KPT, SUBT>;                                                    \
+    set_smem(k, smem);                                                                       \
+    k<<<(unsigned)((g.L + SUBT - 1) / SUBT), kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, \
+                                                                 zero_ptr, zero_words, flag);  \
   }
-  switch (g.R) {
-    case 8: MS_K1(8) break;
-    case 16: MS_K1(16) break;
-    default: MS_K1(32) break;
+  switch (g.R) {  // 16 keys per thread; T = 2048 tiles are counted two per CTA
+    case 8: MS_K1(16, 2) break;
+    case 16: MS_K1(16, 1) break;
+    default: MS_K1(32, 1) break;
   }
 #undef MS_K1
   return cudaGetLastError();
@@ -143,6 +144,7 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   switch (p->kkind) {
     case LOWBITS: return launch_k1<LOWBITS>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case SHIFTC: return launch_k1<SHIFTC>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case SHIFT: return launch_k1<SHIFT>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case DELTA: return launch_k1<DELTA>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case SPLITTERS: return launch_k1<SPLITTERS>(p, g, keys, ids, n, H, zp, zw, flag, s);
     default: return launch_k1<IDS>(p, g, keys, ids, n, H, zp, zw, flag, s);
@@ -164,11 +166,12 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                         uint32_t *vo, uint32_t n, cudaStream_t s) {
   K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
-            p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, &p->bp, sm_count(), s};
+            p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, sm_count(), s};
   if (p->spec.m <= 32) {  // persistent blocked-rank K3 (ms_k3_blocked.cuh), one TU per kind
     switch (p->kkind) {
       case LOWBITS: return k3p_launch_lowbits(a);
       case SHIFTC: return k3p_launch_shiftc(a);
+      case SHIFT: return k3p_launch_shift(a);
       case DELTA: return k3p_launch_delta(a);
       case SPLITTERS: return k3p_launch_splitters(a);
       default: return k3p_launch_ids(a);
@@ -177,6 +180,7 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   switch (p->kkind) {  // m > 32: warp-ballot K3 (ms_k3_warp.cuh)
     case LOWBITS: return k3w_launch_lowbits(a);
     case SHIFTC: return k3w_launch_shiftc(a);
+    case SHIFT: return k3w_launch_shift(a);
     case DELTA: return k3w_launch_delta(a);
     case SPLITTERS: return k3w_launch_splitters(a);
     default: return k3w_launch_ids(a);
@@ -243,8 +247,9 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
     case MS_DELTA:
       if (spec->delta < 1) return MS_ERR_INVALID_ARG;
       if ((spec->delta & (spec->delta - 1)) == 0) {  // power of two (incl. 1): a shift
-        kkind = SHIFTC;
         bp.shift = ceil_log2(spec->delta);
+        // m * delta >= 2^32: k >> shift < m for every key, the clamp is dead
+        kkind = ((uint64_t)m << bp.shift) >= (1ull << 32) ? SHIFT : SHIFTC;
       } else {
         kkind = DELTA;
         const uint64_t c = delta_magic(spec->delta);
@@ -277,10 +282,14 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->bp = bp;
   p->kkind = kkind;
   p->last_launches = 0;
+  // K3 CTA size (m <= 32), measured per workload: 256 threads
+  // (T = 4096) for m > 16 with one-instruction ids, 128 (T = 2048) otherwise
+  p->k3nt = (m > 16 && (kkind == SHIFT || kkind == SHIFTC || kkind == LOWBITS)) ? 256u : 128u;
   // ablation overrides: MS_DEBUG_K3=1 drops K3's global stores;
   // MS_K3_REVERSE=1 walks K3's tiles last-to-first
   if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
   if (const char *e = getenv("MS_K3_REVERSE")) p->bp.reverse = atoi(e) ? 1u : 0u;
+  if (const char *e = getenv("MS_K3_NT")) p->k3nt = atoi(e) == 128 ? 128u : 256u;
   *plan = p;
   return MS_OK;
 }
@@ -495,6 +504,7 @@ ms_status ms_bucket_ids(ms_plan_t p, const uint32_t *keys_in, uint64_t n, uint32
   switch (p->kkind) {
     case LOWBITS: k_bucket_ids<LOWBITS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
     case SHIFTC: k_bucket_ids<SHIFTC><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
+    case SHIFT: k_bucket_ids<SHIFT><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
     case DELTA: k_bucket_ids<DELTA><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
     default: k_bucket_ids<SPLITTERS><<<grid, kThreads, 0, s>>>(keys_in, n, out_ids, p->bp); break;
   }

@@ -9,8 +9,10 @@
 namespace ms {
 
 // Kernel-level bucket-function kinds.  The public kinds (ms.h) map onto
-// these; MS_DELTA becomes SHIFTC when delta is a power of two (incl. 1).
-enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3, SHIFTC = 4 };
+// these; MS_DELTA becomes SHIFTC when delta is a power of two (incl. 1), and
+// SHIFT when in addition m * delta >= 2^32 (the clamp can never fire: the
+// paper's "buckets equally divide the 32-bit domain").
+enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3, SHIFTC = 4, SHIFT = 5 };
 
 constexpr int kThreads = 256;  // CTA = 8 warps (the paper's NW = 8)
 constexpr int kWarps = kThreads / 32;
@@ -71,6 +73,7 @@ template <int KIND>
 __device__ __forceinline__ uint32_t bucket_of_key(uint32_t k, const BucketParams &p,
                                                   const uint32_t *spl_s) {
   if constexpr (KIND == LOWBITS) return id_lowbits(k, p);
+  else if constexpr (KIND == SHIFT) return k >> p.shift;  // m * delta >= 2^32: always < m
   else if constexpr (KIND == SHIFTC) return id_shiftc(k, p);
   else if constexpr (KIND == DELTA) return id_delta(k, p);
   else if constexpr (KIND == SPLITTERS) return id_splitters(k, spl_s, p.logm);

@@ -30,14 +30,14 @@
 
 namespace ms {
 
-template <int LOGMP, bool KV, bool IDS8, int KPT>
+template <int LOGMP, bool KV, bool IDS8, int KPT, int NT = kThreads>
 struct K3pLayout {
   static constexpr int MP = 1 << LOGMP;        // bucket rows (m rounded up to a power of 2, >= 2)
   static constexpr int K = KPT;                // keys per thread (16 or 32)
   static constexpr int CH = K / 4;             // 16-byte chunks per thread per array
-  static constexpr int T = kThreads * K;       // keys per tile
+  static constexpr int T = NT * K;             // keys per tile (NT threads per CTA)
   static constexpr int STAGES = (KV || K > 16) ? 1 : 2;  // tiles prefetched ahead
-  static constexpr int CW = MP * 128;          // counter words (MP x 256 u16)
+  static constexpr int CW = MP * NT / 2;       // counter words (MP x NT u16)
   static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // key slots incl. alignment padding
   static constexpr int WPT = MP / 2;           // counter words per thread in the scan
   static constexpr int MW = 3 * MP + 8;        // per-tile metadata words: rowS[MP+4] P[MP] G[MP]
@@ -73,54 +73,69 @@ __device__ __forceinline__ void cp_async_wait() {
 // Stage this thread's chunks of tile `tile` (keys: CH x 16 B; vals likewise;
 // u8 ids: K/16 x 16 B) into stage slot `st`, chunk-major ([c][tid]) so the
 // later 128-bit reads are conflict-free.  Bytes past n are zero-filled.
-template <bool KV, bool IDS8, int T, int K>
+// owner thread of block beta (inverse of beta(t) = 2*lane + (warp & 1) + 64*(warp >> 1))
+__device__ __forceinline__ uint32_t k3p_owner(uint32_t beta) {
+  const uint32_t lane = (beta >> 1) & 31u, warp = ((beta >> 6) << 1) | (beta & 1u);
+  return warp * 32u + lane;
+}
+
+// Copies are COALESCED: thread t fetches the tile's 16-byte chunks t, t+256,
+// ... (consecutive threads, consecutive chunks -- whole 128-byte lines per
+// warp instruction) and drops chunk g = 4*beta + c (keys 4g..4g+3 of block
+// beta) at the owner's chunk-major slot [c][owner(beta)].  Owners read their
+// chunks only after the begin-of-tile barrier, and a stage is refilled only
+// after the tile's last barrier, so the cross-thread handoff is ordered.
+template <bool KV, bool IDS8, int T, int K, int NT>
 __device__ __forceinline__ void k3p_prefetch(uint32_t *stk, uint32_t *stv, uint32_t *sti, int st,
                                              const uint32_t *keys, const uint32_t *vals, const void *ids,
-                                             uint64_t tile, uint32_t n, uint32_t beta) {
-  constexpr int CH = K / 4;
+                                             uint64_t tile, uint32_t n, uint32_t /*beta*/) {
+  constexpr int CH = K / 4;                 // chunks per block; the tile has NT*CH chunks
   const uint32_t tid = threadIdx.x;
-  const uint64_t b0 = tile * T + (uint64_t)beta * K;
-  uint32_t *dk = stk + st * T + tid * 4;
-  uint32_t *dv = stv + st * T + tid * 4;
-  uint32_t *di = sti + st * (T / 4) + tid * 4;
-  if (tile * T + T <= n) {
+  const uint64_t t0 = tile * T;
+  const bool full = t0 + T <= n;
 #pragma unroll
-    for (int c = 0; c < CH; ++c) {
-      cp_async16_full(dk + c * kThreads * 4, keys + b0 + 4 * c);
-      if constexpr (KV) cp_async16_full(dv + c * kThreads * 4, vals + b0 + 4 * c);
-    }
-    if constexpr (IDS8) {
-#pragma unroll
-      for (int c = 0; c < K / 16; ++c) cp_async16_full(di + c * kThreads * 4, (const uint8_t *)ids + b0 + 16 * c);
-    }
-  } else {
-#pragma unroll
-    for (int c = 0; c < CH; ++c) {
-      const uint64_t e = b0 + 4 * c;
+  for (int i = 0; i < CH; ++i) {
+    const uint32_t g = i * NT + tid;  // chunk index within the tile
+    const uint32_t beta = g / CH, c = g % CH;
+    const uint32_t dst = (c * NT + k3p_owner(beta)) * 4;
+    const uint64_t e = t0 + 4ull * g;
+    if (full) {
+      cp_async16_full(stk + st * T + dst, keys + e);
+      if constexpr (KV) cp_async16_full(stv + st * T + dst, vals + e);
+    } else {
       const uint32_t bytes = e >= n ? 0u : (uint32_t)(umin64(4, n - e) * 4);
       const uint64_t src = bytes ? e : 0;
-      cp_async16(dk + c * kThreads * 4, keys + src, bytes);
-      if constexpr (KV) cp_async16(dv + c * kThreads * 4, vals + src, bytes);
+      cp_async16(stk + st * T + dst, keys + src, bytes);
+      if constexpr (KV) cp_async16(stv + st * T + dst, vals + src, bytes);
     }
-    if constexpr (IDS8) {
+  }
+  if constexpr (IDS8) {  // u8 ids: block beta's K bytes = K/16 chunks, chunk-major by owner
 #pragma unroll
-      for (int c = 0; c < K / 16; ++c) {
-        const uint64_t e = b0 + 16 * c;
+    for (int i = 0; i < K / 16; ++i) {
+      const uint32_t g = i * NT + tid;
+      const uint32_t beta = g / (K / 16), c = g % (K / 16);
+      uint32_t *d = sti + st * (T / 4) + (c * NT + k3p_owner(beta)) * 4;
+      const uint64_t e = t0 + 16ull * g;
+      if (full) {
+        cp_async16_full(d, (const uint8_t *)ids + e);
+      } else {
         const uint32_t bytes = e >= n ? 0u : (uint32_t)umin64(16, n - e);
-        cp_async16(di + c * kThreads * 4, (const uint8_t *)ids + (bytes ? e : 0), bytes);
+        cp_async16(d, (const uint8_t *)ids + (bytes ? e : 0), bytes);
       }
     }
   }
 }
 
 // One tile, already staged.  FULL: all T keys valid (no per-key predicates).
-template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, bool FULL>
+template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, int NT, bool FULL>
 __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *sm_v, const uint32_t *sm_i,
                                          const void *__restrict__ ids, uint32_t *__restrict__ keys_out,
                                          uint32_t *__restrict__ vals_out, uint64_t base, uint32_t nt,
                                          const BucketParams &p, uint32_t *sm, uint32_t beta, uint32_t *meta) {
-  using Ly = K3pLayout<LOGMP, KV, IDS8, KPT>;
+  using Ly = K3pLayout<LOGMP, KV, IDS8, KPT, NT>;
   constexpr int MP = Ly::MP, K = Ly::K, CH = Ly::CH;
+  constexpr int NW = NT / 32;
+  constexpr int LOGNT = NT == 256 ? 8 : 7;
   // ids are recomputed from the key where that is cheaper than keeping them
   constexpr bool KEEP_ID = (KIND == SPLITTERS) || (KIND == IDS && !IDS8);
   uint32_t *cnt32 = sm + Ly::O_CNT;
@@ -134,14 +149,14 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t m = p.m;
   const uint32_t b0 = beta * K;
-  // this thread's counter column: byte address of c[0][beta]; c[j][beta] is j*512 bytes further
+  // this thread's counter column: byte address of c[0][beta]; c[j][beta] is j*2*NT bytes further
   uint8_t *cb = reinterpret_cast<uint8_t *>(cnt32) + 2 * beta;
 
   // Keys (and values) are read from this thread's own staged chunks twice --
   // for counting and again for the scatter -- instead of being held in
   // registers across the scan (no spills at 3 CTAs/SM).
   auto chunk = [&](const uint32_t *st, int c) -> uint4 {
-    return *reinterpret_cast<const uint4 *>(st + (c * kThreads + tid) * 4);
+    return *reinterpret_cast<const uint4 *>(st + (c * NT + tid) * 4);
   };
   uint32_t idw[IDS8 ? K / 4 : 1];
   if constexpr (IDS8) {
@@ -160,11 +175,11 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
     }
   };
 
-  // ---- 1. sequential per-block counting: the rank within the block.
-  // Groups of 4 keys (one staged chunk): the 4 counter loads are issued
-  // together and equal ids inside the group are corrected by compares, so
-  // the read-modify-write chain through shared memory is 4 keys deep
-  // instead of 1.  Keys past the tail (partial tile only) are skipped.
+  // ---- 1. sequential per-block counting: the rank within the block, by an
+  // in-order read-modify-write of the thread's private counter column in
+  // shared memory.  Keys past the tail (partial tile only) are skipped.
+  // (Measured alternatives: a register histogram for m <= 8 and
+  // grouped counter loads with compare corrections were both slower.)
   uint32_t rk[K / 4];                        // ranks (< K), one byte each
   uint32_t idk[KEEP_ID ? K / 4 : 1];         // kept ids, one byte each
   uint4 kx[CH];  // all staged chunks first: no chunk load waits behind a counter store
@@ -180,18 +195,18 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
       id[j] = id_of(kk[j], 4 * c + j);
       ok[j] = FULL || (b0 + 4 * c + j < nt);
     }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) r[j] = ok[j] ? *reinterpret_cast<const uint16_t *>(cb + (id[j] << 9)) : 0u;
-#pragma unroll
-    for (int j = 1; j < 4; ++j)
-#pragma unroll
-      for (int i = 0; i < j; ++i) r[j] += (ok[i] && id[i] == id[j]) ? 1u : 0u;
     rk[c] = 0u;
     if constexpr (KEEP_ID) idk[c] = 0u;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       if (ok[j]) {
-        *reinterpret_cast<uint16_t *>(cb + (id[j] << 9)) = (uint16_t)(r[j] + 1);
+        uint16_t *cp = reinterpret_cast<uint16_t *>(cb + id[j] * (2 * NT));
+        if (p.dbg != 7 && p.dbg != 8) {
+          r[j] = *cp;
+          *cp = (uint16_t)(r[j] + 1);
+        } else {
+          r[j] = 0u;  // ablation: no counting
+        }
         rk[c] |= r[j] << (8 * j);
         if constexpr (KEEP_ID) idk[c] |= id[j] << (8 * j);
       }
@@ -203,7 +218,7 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   // Thread t owns words [t*WPT, (t+1)*WPT) (one bucket row).  With >= 2
   // 16-byte chunks per thread, the chunk order is rotated per lane so the
   // 128-bit accesses of every 8-lane phase hit 8 different bank groups.
-  const uint32_t row = tid >> (8 - LOGMP);
+  const uint32_t row = tid >> (LOGNT - LOGMP);
   constexpr int WPT = Ly::WPT;
   constexpr int NC = WPT >= 4 ? WPT / 4 : 1;       // 16-byte chunks per thread
   constexpr int CWD = WPT >= 4 ? 4 : WPT;          // words per chunk
@@ -214,7 +229,10 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   for (int i = 0; i < NC; ++i) {
     const uint32_t pc = (i + rot) & (NC - 1);   // physical chunk held in register slot i
     const uint32_t *src = cnt32 + tid * WPT + pc * CWD;
-    if constexpr (CWD == 4) {
+    if (p.dbg >= 6 && p.dbg <= 8) {  // ablation: no scan traffic
+#pragma unroll
+      for (int j = 0; j < CWD; ++j) w[i][j] = 0u;
+    } else if constexpr (CWD == 4) {
       const uint4 x = *reinterpret_cast<const uint4 *>(src);
       w[i][0] = x.x; w[i][1] = x.y; w[i][2] = x.z; w[i][3] = x.w;
     } else if constexpr (CWD == 2) {
@@ -236,13 +254,13 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   __syncthreads();
   uint32_t wpre = 0, tot = 0;
 #pragma unroll
-  for (int i = 0; i < kWarps; ++i) {
+  for (int i = 0; i < NW; ++i) {
     const uint32_t x = wsum[i];
     wpre += (i < (int)warp) ? x : 0u;
     tot += x;
   }
   const uint32_t excl = wpre + incl - s;
-  constexpr uint32_t TPR = kThreads >> LOGMP;  // threads per bucket row
+  constexpr uint32_t TPR = NT >> LOGMP;  // threads per bucket row
   // S_row = excl of the row's first thread: a lane of this warp (rows < 32
   // threads) or lane 0 of warp row*TPR/32, whose excl is the warp prefix.
   uint32_t Sr;
@@ -252,7 +270,7 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
     Sr = 0;
     const uint32_t w0 = (row * TPR) >> 5;
 #pragma unroll
-    for (int i = 0; i < kWarps; ++i) Sr += ((uint32_t)i < w0) ? wsum[i] : 0u;
+    for (int i = 0; i < NW; ++i) Sr += ((uint32_t)i < w0) ? wsum[i] : 0u;
   }
   if ((tid & (TPR - 1)) == 0) rowS[row] = excl;
   if (tid == 0) rowS[MP] = tot;
@@ -270,10 +288,11 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
     for (int j = 0; j < CWD; ++j) {
       const uint32_t x = w[i][j];
       w[i][j] = run * 0x10001u + (x << 16);      // (run, run + lo)
-      run += (x & 0xFFFFu) + (x >> 16);
+      run += (x * 0x10001u) >> 16;               // lo + hi (< 2^16, no carry into bit 32)
     }
     uint32_t *dst = cnt32 + tid * WPT + pc * CWD;
-    if constexpr (CWD == 4) *reinterpret_cast<uint4 *>(dst) = make_uint4(w[i][0], w[i][1], w[i][2], w[i][3]);
+    if (p.dbg >= 6 && p.dbg <= 8) {
+    } else if constexpr (CWD == 4) *reinterpret_cast<uint4 *>(dst) = make_uint4(w[i][0], w[i][1], w[i][2], w[i][3]);
     else if constexpr (CWD == 2) *reinterpret_cast<uint2 *>(dst) = make_uint2(w[i][0], w[i][1]);
     else dst[0] = w[i][0];
   }
@@ -304,14 +323,14 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
       uint32_t id;
       if constexpr (KEEP_ID) id = __byte_perm(idk[c], 0u, 0x4440u + j);
       else id = id_of(kk[j], q);
-      sl[j] = (FULL || b0 + q < nt) ? *reinterpret_cast<const uint16_t *>(cb + (id << 9)) : 0u;
+      sl[j] = (FULL || b0 + q < nt) ? *reinterpret_cast<const uint16_t *>(cb + id * (2 * NT)) : 0u;
     }
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       const int q = 4 * c + j;
       if (FULL || b0 + q < nt) {
         const uint32_t slot = sl[j] + __byte_perm(rk[c], 0u, 0x4440u + j);
-        keys_s[slot] = kk[j];
+        if (p.dbg != 8) keys_s[slot] = kk[j];
         if constexpr (KV) vals_s[slot] = vv[j];
       }
     }
@@ -319,38 +338,54 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA (async proxy)
   __syncthreads();
 
-  // ---- 4. bucket runs: 8 threads per bucket -- 3 head keys, 3 tail keys,
-  //         and the TMA bulk store(s) of the 16-byte-aligned body
-  if (p.dbg == 1) return;  // ablation: no stores
+  // ---- 4. bucket runs: NT/32 threads per bucket (m <= 32) share its
+  //         <= 3 head keys, <= 3 tail keys and the TMA bulk store(s) of the
+  //         16-byte-aligned body
+  if (p.dbg == 1 || (p.dbg >= 6 && p.dbg <= 8)) return;  // ablation: no stores
   {
-    const uint32_t b = tid >> 3, sub = tid & 7;
+    constexpr uint32_t SPB = NT / 32;
+    const uint32_t b = tid / SPB, sub = tid % SPB;
     if (b < m) {
       const uint32_t len = rowS[b + 1] - rowS[b];
       const uint32_t P = Pj[b], Gd = Gj[b];
       const uint32_t head = min(len, (4u - (Gd & 3u)) & 3u);
       const uint32_t body = (len - head) & ~3u;
-      if (sub < 6) {
-        const uint32_t i = sub < 3 ? sub : head + body + (sub - 3);
-        if ((sub < 3 && sub < head) || (sub >= 3 && i < len)) {
-          keys_out[Gd + i] = keys_s[P + i];
-          if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+      if constexpr (SPB == 8) {
+        if (sub < 6) {
+          const uint32_t i = sub < 3 ? sub : head + body + (sub - 3);
+          if ((sub < 3 && sub < head) || (sub >= 3 && i < len)) {
+            keys_out[Gd + i] = keys_s[P + i];
+            if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+          }
+        } else if (body) {
+          if (sub == 6) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
+          else if (KV) bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
+          bulk_commit();
         }
-      } else if (body) {
-        if (sub == 6) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
-        else if (KV) bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
-        bulk_commit();
+      } else {  // SPB == 4: head / tail / keys body / values body
+        if (sub < 2) {
+          const uint32_t i0 = sub == 0 ? 0u : head + body, i1 = sub == 0 ? head : len;
+          for (uint32_t i = i0; i < i1; ++i) {
+            keys_out[Gd + i] = keys_s[P + i];
+            if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+          }
+        } else if (body) {
+          if (sub == 2) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
+          else if (KV) bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
+          bulk_commit();
+        }
       }
     }
   }
 }
 
-template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT>
-__global__ void __launch_bounds__(kThreads, (KV || KPT > 16) ? 2 : 3)
+template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, int NT>
+__global__ void __launch_bounds__(NT, NT == 256 ? (KV ? 2 : 3) : (KV ? 4 : 6))
 k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const void *__restrict__ ids, const uint32_t *__restrict__ G,
              uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
              uint32_t L, const __grid_constant__ BucketParams p) {
-  using Ly = K3pLayout<LOGMP, KV, IDS8, KPT>;
+  using Ly = K3pLayout<LOGMP, KV, IDS8, KPT, NT>;
   constexpr int T = Ly::T, STAGES = Ly::STAGES, CW = Ly::CW, MP = Ly::MP, K = Ly::K;
   extern __shared__ __align__(128) uint32_t sm[];
   uint32_t *stk = sm + Ly::O_STK;
@@ -382,7 +417,7 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   // prologue: STAGES tiles in flight
 #pragma unroll
   for (int s = 0; s < STAGES; ++s) {
-    if ((uint32_t)s < iters) k3p_prefetch<KV, IDS8, T, K>(stk, stv, sti, s, keys, vals, ids, tile_of(s), n, beta);
+    if ((uint32_t)s < iters) k3p_prefetch<KV, IDS8, T, K, NT>(stk, stv, sti, s, keys, vals, ids, tile_of(s), n, beta);
     cp_async_commit();
   }
   uint32_t gnext = 0;
@@ -392,11 +427,13 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   // tile's scatter, before a barrier), publish G[:, tile] into this parity's
   // metadata, prefetch the next G column, wait for this thread's staged chunks
   auto begin_tile = [&](uint32_t it, uint32_t *meta) {
-    uint4 *c4 = reinterpret_cast<uint4 *>(sm + Ly::O_CNT);
+    {
+      uint4 *c4 = reinterpret_cast<uint4 *>(sm + Ly::O_CNT);
 #pragma unroll
-    for (int i = 0; i < (CW / 4 + kThreads - 1) / kThreads; ++i) {
-      const int idx = i * kThreads + tid;
-      if (idx < CW / 4) c4[idx] = make_uint4(0, 0, 0, 0);
+      for (int i = 0; i < (CW / 4 + NT - 1) / NT; ++i) {
+        const int idx = i * NT + tid;
+        if (idx < CW / 4) c4[idx] = make_uint4(0, 0, 0, 0);
+      }
     }
     if (tid < m) meta[MP + 4 + MP + tid] = gnext;
     if (it + 1 < iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(it + 1));
@@ -409,9 +446,9 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const uint64_t tile = tile_of(0);
     uint32_t *meta = sm + Ly::O_META;
     begin_tile(0, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, false>(stk, stv, sti, ids, keys_out, vals_out, tile * T,
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, false>(stk, stv, sti, ids, keys_out, vals_out, tile * T,
                                                 (uint32_t)(n - tile * T), p, sm, beta, meta);
-    if (STAGES < iters) k3p_prefetch<KV, IDS8, T, K>(stk, stv, sti, 0, keys, vals, ids, tile_of(STAGES), n, beta);
+    if (STAGES < iters) k3p_prefetch<KV, IDS8, T, K, NT>(stk, stv, sti, 0, keys, vals, ids, tile_of(STAGES), n, beta);
     cp_async_commit();
     it = 1;
   }
@@ -420,11 +457,11 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const int st = (int)(it % STAGES);
     uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
     begin_tile(it, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, true>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, true>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
                                                vals_out, tile * T, T, p, sm, beta, meta);
     // refill this stage with tile it + STAGES (own chunks only; already consumed)
     if (it + STAGES < iters)
-      k3p_prefetch<KV, IDS8, T, K>(stk, stv, sti, st, keys, vals, ids, tile_of(it + STAGES), n, beta);
+      k3p_prefetch<KV, IDS8, T, K, NT>(stk, stv, sti, st, keys, vals, ids, tile_of(it + STAGES), n, beta);
     cp_async_commit();
   }
   if (has_tail) {
@@ -432,31 +469,39 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const int st = (int)(it % STAGES);
     uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
     begin_tile(it, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, false>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, false>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
                                                 vals_out, tile * T, (uint32_t)(n - tile * T), p, sm, beta, meta);
   }
   bulk_wait_read0();
 }
 
 // ------------------------------------------------------------------ host launcher
-template <typename Kern>
+template <int NT, typename Kern>
 inline cudaError_t k3p_launch_one(Kern k, size_t smem, const K3pArgs &a) {
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, NT, smem);
   if (per_sm <= 0) per_sm = 1;
+  if (a.bp->dbg >= 10 && (int)(a.bp->dbg - 10) < per_sm) per_sm = (int)(a.bp->dbg - 10);  // ablation: CTAs/SM
   const unsigned grid = (unsigned)umin64_host(a.L, (uint64_t)a.sms * per_sm);
-  k<<<grid, kThreads, smem, a.stream>>>(a.keys, a.vals, a.ids, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+  k<<<grid, NT, smem, a.stream>>>(a.keys, a.vals, a.ids, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
   return cudaGetLastError();
+}
+
+template <int KIND, bool KV, int LOGMP, int KPT, int NT>
+inline cudaError_t k3p_launch_n(const K3pArgs &a) {
+  if constexpr (KIND == IDS) {
+    if (a.id_bytes == 1)
+      return k3p_launch_one<NT>(k3p_postscan<KIND, KV, LOGMP, true, KPT, NT>,
+                                K3pLayout<LOGMP, KV, true, KPT, NT>::BYTES, a);
+  }
+  return k3p_launch_one<NT>(k3p_postscan<KIND, KV, LOGMP, false, KPT, NT>,
+                            K3pLayout<LOGMP, KV, false, KPT, NT>::BYTES, a);
 }
 
 template <int KIND, bool KV, int LOGMP, int KPT>
 inline cudaError_t k3p_launch_l(const K3pArgs &a) {
-  if constexpr (KIND == IDS) {
-    if (a.id_bytes == 1)
-      return k3p_launch_one(k3p_postscan<KIND, KV, LOGMP, true, KPT>, K3pLayout<LOGMP, KV, true, KPT>::BYTES, a);
-  }
-  return k3p_launch_one(k3p_postscan<KIND, KV, LOGMP, false, KPT>, K3pLayout<LOGMP, KV, false, KPT>::BYTES, a);
+  return a.nt == 128 ? k3p_launch_n<KIND, KV, LOGMP, KPT, 128>(a) : k3p_launch_n<KIND, KV, LOGMP, KPT, 256>(a);
 }
 
 template <int KIND, bool KV, int KPT>

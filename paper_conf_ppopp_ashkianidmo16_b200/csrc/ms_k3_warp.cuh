@@ -30,7 +30,7 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
                                         uint32_t *gD_s, const uint32_t *spl_s, uint8_t *id8_s,
                                         uint32_t *wsum, uint32_t gcol) {
   constexpr int SEG = 32 * R;
-  constexpr bool ID8 = (KIND != LOWBITS && KIND != SHIFTC);
+  constexpr bool ID8 = (KIND != LOWBITS && KIND != SHIFTC && KIND != SHIFT);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t m = p.m;
   const uint32_t lt = lanemask_lt(), gt = lanemask_gt();
@@ -201,7 +201,7 @@ inline size_t k3w_smem(int R, bool kv, bool id8) {
 
 template <int KIND, bool KV, int R, int LOGM>
 inline cudaError_t k3w_launch_l(const K3pArgs &a) {
-  constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC);
+  constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC && KIND != SHIFT);
   auto k = k3_postscan<KIND, KV, R, LOGM>;
   const size_t smem = k3w_smem(R, KV, id8);
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

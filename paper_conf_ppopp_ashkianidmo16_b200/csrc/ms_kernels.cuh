@@ -25,20 +25,25 @@ __device__ __forceinline__ uint32_t k1_slot(uint32_t tid) {
   return (warp >> 2) * 128 + lane * 4 + (warp & 3);
 }
 
-template <int KIND, int KPT>
+template <int KIND, int KPT, int SUBT>
 __global__ void __launch_bounds__(kThreads)
 k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
            uint32_t L, uint32_t *__restrict__ H, const __grid_constant__ BucketParams p,
            uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
-  constexpr int T = kThreads * KPT;
+  // SUBT tiles per CTA: warps [h*8/SUBT, (h+1)*8/SUBT) count tile SUBT*blockIdx + h.
+  // The byte-counter slot layout puts warps 0-3 in bytes [0,128) of every row and
+  // warps 4-7 in [128,256), so each half-row is one tile's column.
+  constexpr int NTS = kThreads / SUBT;   // threads per tile
+  constexpr int T = NTS * KPT;           // keys per tile
   static_assert(KPT <= 255 && KPT % 4 == 0, "byte counters");
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t *spl_s = smem;                                     // kMaxM words (SPLITTERS)
   uint8_t *c8 = reinterpret_cast<uint8_t *>(smem + kMaxM);    // [m][256] bytes
   const uint32_t tid = threadIdx.x, lane = tid & 31;
-  const uint32_t tile = blockIdx.x;
-  const uint64_t base = (uint64_t)tile * T;
-  const uint32_t nt = (uint32_t)umin64(T, n - base);
+  const uint32_t h = tid / NTS, tl = tid % NTS;
+  const uint64_t tile = (uint64_t)blockIdx.x * SUBT + h;
+  const uint64_t base = tile * T;
+  const uint32_t nt = tile < L ? (uint32_t)umin64(T, n - base) : 0u;
   const uint32_t m = p.m;
 
   // issue this thread's loads first (they overlap the shared-memory setup)
@@ -47,10 +52,10 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   if (full) {
     const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
 #pragma unroll
-    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * kThreads + tid);  // cached: K3 reuses the tail from L2
+    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * NTS + tl);  // coalesced 128-bit loads
   }
   // K2's look-back status words are cleared here (K1 precedes K2 in the stream).
-  for (uint32_t i = tile * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
+  for (uint32_t i = blockIdx.x * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
   uint4 *c4 = reinterpret_cast<uint4 *>(c8);
   for (uint32_t i = tid; i < m * 16; i += kThreads) c4[i] = make_uint4(0, 0, 0, 0);
   if constexpr (KIND == SPLITTERS) {
@@ -64,7 +69,7 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
     if constexpr (KIND == IDS) {
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) {
-        const uint64_t i0 = base + 4ull * (j * kThreads + tid);
+        const uint64_t i0 = base + 4ull * (j * NTS + tl);
         uint32_t raw[4];
         if (p.id_bytes == 1) {
           uint32_t w = __ldg(reinterpret_cast<const uint32_t *>((const uint8_t *)ids + i0));
@@ -89,7 +94,7 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
       }
     }
   } else {
-    for (uint32_t i = tid; i < nt; i += kThreads) {
+    for (uint32_t i = tl; i < nt; i += NTS) {
       uint32_t id;
       if constexpr (KIND == IDS) {
         uint32_t raw = p.id_bytes == 1 ? (uint32_t)((const uint8_t *)ids)[base + i]
@@ -107,19 +112,22 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   }
   __syncthreads();
 
-  // row j = bucket j's 256 byte counters; thread j sums it
-  if (tid < m) {
-    const uint4 *row = c4 + tid * 16;
+  // tile column j = the bytes of row j that belong to this tile's threads;
+  // thread j (< m) of each half sums its 256/SUBT bytes with dp4a, reading
+  // 16-byte chunks in a lane-rotated order (conflict-free)
+  constexpr int CPH = 16 / SUBT;  // 16-byte chunks per half-row
+  for (uint32_t b = tl; b < m && tile < L; b += NTS) {
+    const uint4 *row = c4 + b * 16 + h * CPH;
     uint32_t acc = 0;
 #pragma unroll
-    for (int j = 0; j < 16; ++j) {
-      const uint4 w = row[(j + tid) & 15];
+    for (int j = 0; j < CPH; ++j) {
+      const uint4 w = row[(j + b) & (CPH - 1)];
       acc = __dp4a(w.x, 0x01010101u, acc);
       acc = __dp4a(w.y, 0x01010101u, acc);
       acc = __dp4a(w.z, 0x01010101u, acc);
       acc = __dp4a(w.w, 0x01010101u, acc);
     }
-    H[(uint64_t)tid * L + tile] = acc;
+    H[(uint64_t)b * L + tile] = acc;
   }
 }
 
