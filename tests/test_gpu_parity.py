@@ -171,6 +171,51 @@ def test_splitter_functor_dense():
         assert np.array_equal(got, exp.astype(np.uint32))
 
 
+def _clustered_splitter_sets():
+    """Splitter sets that stress the top-byte table: crowded 2^24 windows (fallback
+    search), splitters exactly on window boundaries, at 0 / 2^32-1, and duplicates."""
+    rng = np.random.default_rng(11)
+    sets = []
+    for m in (2, 5, 32, 33, 200, 256):
+        sets.append(sorted(int(x) for x in rng.integers(0x37000000, 0x37001000, m - 1)))   # one window
+        sets.append(sorted(int(t) << 24 for t in rng.integers(0, 256, m - 1)))             # boundaries
+        half = (m - 1) // 2
+        mix = [int(x) for x in rng.integers(0, 1 << 32, half)] + [0xA0FFFFFF] * ((m - 1) - half)
+        sets.append(sorted(mix))
+    sets.append([0])
+    sets.append([0xFFFFFFFF])
+    sets.append([0, 0xFFFFFFFF, 0xFFFFFFFF])
+    return sets
+
+
+def test_splitter_functor_clustered():
+    P = _pkg()
+    for spl in _clustered_splitter_sets():
+        near = {s + d for s in spl for d in (-1, 0, 1) if 0 <= s + d <= 0xFFFFFFFF}
+        near |= {(t << 24) + d for t in range(256) for d in (-1, 0, 1) if 0 <= (t << 24) + d <= 0xFFFFFFFF}
+        kn = np.array(sorted(near | {0xFFFFFFFF}), dtype=np.uint32)
+        plan = P.Plan(P.BucketSpec.from_splitters(spl), len(kn))
+        got = from_dev(plan.bucket_ids(to_dev(kn)))
+        exp = np.searchsorted(np.array(spl, dtype=np.uint64), kn.astype(np.uint64), side="left")
+        assert np.array_equal(got, exp.astype(np.uint32)), f"m={len(spl) + 1}"
+
+
+def test_parity_clustered_splitters():
+    """Full K1/K2/K3 pipeline with clustered splitters, keys drawn near the splitters."""
+    for i, spl in enumerate(_clustered_splitter_sets()):
+        m = len(spl) + 1
+        rng = np.random.default_rng(100 + i)
+        n = 70001
+        base = np.array(spl, dtype=np.int64)[rng.integers(0, len(spl), n)]
+        keys = np.clip(base + rng.integers(-3000, 3000, n), 0, 0xFFFFFFFF).astype(np.uint32)
+        keys[::7] = W.keys_np(n, i)[::7]
+        for kv in (False, True):
+            vals = W.values_np(n, i, "index") if kv else None
+            case = dict(spec_kw=dict(kind="splitters", m=m, splitters=spl), keys=keys, vals=vals, ids=None,
+                        ospec=oracle.Spec("splitters", m, splitters=spl))
+            _assert_equal(case, _run_case(case), _expect(case), f"clustered set {i} m={m} kv={kv}")
+
+
 def test_validate_flags_out_of_range_ids():
     P = _pkg()
     n, m = 10000, 16
