@@ -4,8 +4,8 @@
 Contract (one JSON line from rank 0):
   python bench.py --gpus N --steps K --warmup W [--impl ours|reference] [--config C2]
 
-A step = one whole multisplit (K1 pre-scan -> K2 scan -> K3 post-scan, or the
-one-pass variant) over the config's synthetic input, already resident in HBM.
+A step = one whole multisplit (K1 pre-scan -> K2 scan -> K3 post-scan, in the
+plan's tile or CTA-range variant) over the config's synthetic input, already resident in HBM.
 L2 is flushed (a 512 MiB write) between timed steps, outside the timed
 kernels.  Timing = CUDA events recorded by libms's native per-stage trace on
 the launch stream; max over ranks.  `e2e` = the same metric through
@@ -267,7 +267,12 @@ def run_reference(args, cfg, world, rank):
 
 # ------------------------------------------------------------------ our arm
 def measure_device(cfg, plan, keys, vals, K, Wm, flush, device):
-    """Warm up, then K traced runs with an L2 flush between them.  Returns per-run stage times (ms)."""
+    """Warm up, then two passes of K runs, each with an L2 flush before every run:
+    (1) the timed pass: libms records one event before K1 and one after K3 of every
+        run (trace mode "run"; the kernels keep their programmatic dependent launch);
+    (2) the breakdown pass: an event between every two kernels (per-stage times; the
+        kernels then launch without PDL, so these stages sum to slightly more).
+    Returns (per-run whole-step ms, per-run stage ms [k1, k2, k3, total], launches per run)."""
     import torch
     keys_out = torch.empty_like(keys)
     vals_out = torch.empty_like(vals) if vals is not None else None
@@ -276,14 +281,17 @@ def measure_device(cfg, plan, keys, vals, K, Wm, flush, device):
     for _ in range(Wm):
         plan.run(keys, vals, keys_out=keys_out, vals_out=vals_out, offsets=offsets, workspace=ws)
     torch.cuda.synchronize()
-    plan.trace(True)
-    for _ in range(K):
-        flush()
-        plan.run(keys, vals, keys_out=keys_out, vals_out=vals_out, offsets=offsets, workspace=ws)
-    torch.cuda.synchronize()
-    runs = plan.trace_read(K)
-    plan.trace(False)
-    return runs, plan.last_launches()
+    out = []
+    for mode in ("run", True):
+        plan.trace(mode)
+        for _ in range(K):
+            flush()
+            plan.run(keys, vals, keys_out=keys_out, vals_out=vals_out, offsets=offsets, workspace=ws)
+        torch.cuda.synchronize()
+        out.append(plan.trace_read(K))
+        plan.trace(False)
+    whole = [r[3] for r in out[0]]
+    return whole, out[1], plan.last_launches()
 
 
 def measure_e2e(cfg, plan, keys_d, vals_d, K):
@@ -323,10 +331,10 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True):
     barrier(world)
     clocks = ClockSampler(torch.cuda.current_device())
     with clocks:
-        runs, launches = measure_device(cfg, plan, keys, vals, K, Wm, flush, device)
+        whole, runs, launches = measure_device(cfg, plan, keys, vals, K, Wm, flush, device)
     barrier(world)
     runs = np.array(runs, dtype=np.float64)
-    total_ms = float(runs[:, 3].sum())
+    total_ms = float(np.sum(whole))
     total_ms = max_over_ranks(total_ms, world, device)
     ms_step = total_ms / K
     value = n * world / (ms_step * 1e-3) / 1e9
@@ -340,7 +348,8 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True):
     alg_bytes = model.algorithmic_bytes_per_key(cfg["kv"]) * n
     res = {
         "value": value, "ms_per_step": ms_step,
-        "stages_ms": {"k1_prescan": k1_ms, "k2_scan": k2_ms, "k3_postscan": k3_ms},
+        "stages_ms": {"k1_prescan": k1_ms, "k2_scan": k2_ms, "k3_postscan": k3_ms,
+                      "sum_without_pdl": float(runs[:, 3].mean())},
         "whole_step_hbm_gbs": alg_bytes / (ms_step * 1e-3) / 1e9,
         "whole_step_frac": alg_bytes / (ms_step * 1e-3) / 1e9 / peak,
         "roofline": {"bound": "hbm", "kernel": "k3_postscan", "achieved": round(achieved, 1), "peak": peak,

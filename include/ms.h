@@ -15,7 +15,14 @@
  *   K2 scan       G = exclusive scan of row-vectorised H, offsets = G[:,0]
  *   K3 post-scan  recompute ids, stable tile-local multisplit in shared
  *                 memory, coalesced scatter to G[j][l] + local offset
- * or the one-pass variant (global histogram + decoupled look-back).
+ * Two variants (ms_plan_geometry reports which one a plan uses):
+ *   0 "tile"   subproblems = the L tiles (H, G are m x L words);
+ *   1 "ranged" (default for m <= 32) subproblems = the C <= 2048 contiguous
+ *              tile ranges of K3's persistent CTAs: K1 writes per-range
+ *              histograms (m x C), K2 is a one-CTA scan of them, and K3 keeps
+ *              each tile's G_j as a running sum inside its range (Eq. (2)
+ *              applied twice).
+ * The stage-wise calls (ms_prescan / ms_scan / ms_postscan) always use tiles.
  *
  * Conventions for every call below:
  *  - Pointers named *_in/*_out/ids/offsets/workspace/H/G are CUDA DEVICE
@@ -75,8 +82,8 @@ typedef struct ms_plan_s *ms_plan_t;
 
 /* plan flags */
 #define MS_VALIDATE      1u  /* flag precomputed ids >= m on the device; ms_plan_check reports it */
-#define MS_VARIANT_3K    2u  /* force the 3-kernel {pre-scan, scan, post-scan} path              */
-#define MS_VARIANT_1P    4u  /* force the one-pass (histogram + decoupled look-back) path        */
+#define MS_VARIANT_3K     2u  /* force the tile variant (H, G per tile; any m)                   */
+#define MS_VARIANT_RANGED 4u  /* force the ranged variant (m <= 32, else MS_ERR_UNSUPPORTED)      */
 
 /* Create a plan for up to max_n elements (max_n < 2^32).  with_values != 0
  * plans key-value runs.  Host-only: validates the spec (m range, power-of-two
@@ -89,7 +96,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
 ms_status ms_plan_workspace_size(ms_plan_t plan, uint64_t n, size_t *bytes);
 
 /* Tile geometry the plan uses for n elements: tile = T (keys per subproblem),
- * num_tiles = L = ceil(n / T), variant = 0 (3-kernel) or 1 (one-pass). */
+ * num_tiles = L = ceil(n / T), variant = 0 (tile) or 1 (ranged). */
 ms_status ms_plan_geometry(ms_plan_t plan, uint64_t n, uint32_t *tile, uint64_t *num_tiles,
                            int32_t *variant);
 
@@ -148,13 +155,17 @@ int32_t ms_plan_last_launches(ms_plan_t plan);
  * post-scan split).  ms_plan_trace(plan, 1) clears the record
  * and makes every following ms_run record an event before its first kernel
  * and after each kernel on its stream (plan-owned events, created on first
- * use); ms_plan_trace(plan, 0) stops recording.  ms_plan_trace_read waits
+ * use); ms_plan_trace(plan, 2) records only the first and the last event
+ * of every run (no events between the kernels, so K2 and K3 keep their
+ * programmatic dependent launch; stage durations then read 0);
+ * ms_plan_trace(plan, 0) stops recording.  ms_plan_trace_read waits
  * for the recorded events and writes, for up to max_runs runs in order,
  * stage_ms[r * 4 + s] = duration of stage s of run r in milliseconds
- * (3-kernel: s = 0 K1, 1 K2, 2 K3; one-pass: 0 histogram, 1 unused (0),
- * 2 fused pass), and stage_ms[r * 4 + 3] = the run's total; *runs and
+ * (s = 0 K1 pre-scan, 1 K2 scan, 2 K3 post-scan, in either variant),
+ * and stage_ms[r * 4 + 3] = the run's total; *runs and
  * *stages (3) report what was written.  Tracing is host-side bookkeeping
- * only; it adds no kernel launches. */
+ * only; it adds no kernel launches.  With per-stage events (mode 1) the
+ * kernels are launched without programmatic dependent launch. */
 ms_status ms_plan_trace(ms_plan_t plan, int enable);
 ms_status ms_plan_trace_read(ms_plan_t plan, float *stage_ms, int32_t max_runs, int32_t *runs,
                              int32_t *stages);

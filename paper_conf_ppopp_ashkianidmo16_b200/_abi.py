@@ -22,7 +22,7 @@ MS_ERR_CUDA = -6
 MS_ERR_BUCKET_RANGE = -8
 
 MS_LOWBITS, MS_DELTA, MS_SPLITTERS, MS_IDS = 0, 1, 2, 3
-MS_VALIDATE, MS_VARIANT_3K, MS_VARIANT_1P = 1, 2, 4
+MS_VALIDATE, MS_VARIANT_3K, MS_VARIANT_RANGED = 1, 2, 4
 
 # every symbol include/ms.h declares (tests check the library exports them all)
 EXPORTS = [

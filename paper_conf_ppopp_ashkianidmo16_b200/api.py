@@ -88,8 +88,8 @@ class Plan:
         flags = _abi.MS_VALIDATE if validate else 0
         if variant == "3k":
             flags |= _abi.MS_VARIANT_3K
-        elif variant == "1p":
-            flags |= _abi.MS_VARIANT_1P
+        elif variant == "ranged":
+            flags |= _abi.MS_VARIANT_RANGED
         self.spec = spec
         self.max_n = int(max_n)
         self.with_values = bool(with_values)
@@ -135,9 +135,11 @@ class Plan:
     def last_launches(self) -> int:
         return int(_abi.lib().ms_plan_last_launches(self._h))
 
-    def trace(self, enable: bool = True):
-        """ms_plan_trace: record per-stage CUDA events on every following run."""
-        check(_abi.lib().ms_plan_trace(self._h, int(enable)), "ms_plan_trace")
+    def trace(self, enable=True):
+        """ms_plan_trace: record CUDA events on every following run -- per stage
+        (True / 1; kernels then launch without PDL) or whole run only ("run" / 2)."""
+        mode = 2 if enable == "run" else int(bool(enable)) if not isinstance(enable, int) else enable
+        check(_abi.lib().ms_plan_trace(self._h, mode), "ms_plan_trace")
 
     def trace_read(self, max_runs: int = 100000):
         """ms_plan_trace_read -> list of [stage0_ms, stage1_ms, stage2_ms, total_ms] per traced run."""

@@ -16,6 +16,7 @@
 #include "../../include/ms.h"
 #include "ms_kernels.cuh"
 #include "ms_k3p_args.h"
+#include "ms_ranged.cuh"
 
 using namespace ms;
 
@@ -28,9 +29,12 @@ struct ms_plan_s {
   int kkind;  // kernel-level Kind (ms_device.cuh)
   uint32_t kpt = 16;  // K3 (m <= 32): keys per thread
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt (MS_K3_NT)
+  int ranged = 0;  // CTA-range variant (ms_ranged.cuh, m <= 32): 0 never, 1 when L is large, 2 always
+  int pdl = 1;     // programmatic dependent launch of K2, K3 (MS_PDL=0 disables)
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
-  int tracing = 0;
+  int tracing = 0;     // 0 off, 1 per-stage events, 2 whole-run events only
+  int trace_mode = 1;  // mode of the recorded runs (kept after tracing stops)
   size_t trace_runs = 0;
   std::vector<cudaEvent_t> trace_ev;  // 4 * capacity
 };
@@ -83,6 +87,7 @@ struct Geometry {
   uint64_t hg_words;   // m * L
   uint64_t chunks;     // K2 CTAs
   size_t off_hg, off_status, off_flag, bytes;
+  size_t off_hc, off_gb;  // CTA-range variant: HC[C][m], GB[C][m] (C <= kMaxRanges), over the H/G region
 };
 
 Geometry geometry(const ms_plan_s *p, uint64_t n) {
@@ -97,6 +102,13 @@ Geometry geometry(const ms_plan_s *p, uint64_t n) {
   g.off_hg = kAlign;
   g.off_status = g.off_hg + align_up(g.hg_words * 4);
   g.bytes = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);
+  if (p->spec.m <= 32) {  // the range arrays reuse the tile arrays' space (never live together)
+    const size_t hw = align_up((size_t)kMaxRangeRows * p->spec.m * 4);
+    const size_t rw = align_up(std::min<uint64_t>(std::max<uint64_t>(g.L, 1), kMaxRanges) * p->spec.m * 4);
+    g.off_hc = g.off_hg;
+    g.off_gb = g.off_hc + hw;
+    g.bytes = std::max(g.bytes, g.off_gb + rw);
+  }
   return g;
 }
 
@@ -164,9 +176,13 @@ int sm_count() {
 
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
-                        uint32_t *vo, uint32_t n, cudaStream_t s) {
+                        uint32_t *vo, uint32_t n, cudaStream_t s, int ranged = 0,
+                        uint32_t *grid_out = nullptr, int pdl = 0) {
   K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
             p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, sm_count(), s};
+  a.ranged = ranged;
+  a.grid_out = grid_out;
+  a.pdl = pdl;
   if (p->spec.m <= 32) {  // persistent blocked-rank K3 (ms_k3_blocked.cuh), one TU per kind
     switch (p->kkind) {
       case LOWBITS: return k3p_launch_lowbits(a);
@@ -185,6 +201,38 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
     case SPLITTERS: return k3w_launch_splitters(a);
     default: return k3w_launch_ids(a);
   }
+}
+
+// K1r: k sub-ranges per range so that the grid has ~8 CTAs of 256 threads per SM
+uint32_t k1r_split(uint32_t C) {
+  return std::max<uint32_t>(1u, std::min<uint32_t>(8u * (uint32_t)sm_count() / C, kMaxRangeRows / C));
+}
+
+template <int KIND>
+cudaError_t launch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, const uint32_t *keys, const void *ids,
+                       uint32_t n, uint32_t *HC, uint32_t *flag, cudaStream_t s) {
+  const uint32_t k = k1r_split(C);
+  auto kern = k1r_prescan<KIND, 256>;
+  const size_t smem = k1r_smem(p->spec.m, KIND, 256);
+  set_smem(kern, smem);
+  kern<<<C * k, 256, smem, s>>>(keys, ids, n, (uint32_t)g.L, g.T, C, k, HC, p->bp, flag);
+  return cudaGetLastError();
+}
+
+cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, const uint32_t *keys, const void *ids,
+                         uint32_t n, uint32_t *HC, uint32_t *flag, cudaStream_t s) {
+  switch (p->kkind) {
+    case LOWBITS: return launch_k1r<LOWBITS>(p, g, C, keys, ids, n, HC, flag, s);
+    case SHIFTC: return launch_k1r<SHIFTC>(p, g, C, keys, ids, n, HC, flag, s);
+    case SHIFT: return launch_k1r<SHIFT>(p, g, C, keys, ids, n, HC, flag, s);
+    case DELTA: return launch_k1r<DELTA>(p, g, C, keys, ids, n, HC, flag, s);
+    case SPLITTERS: return launch_k1r<SPLITTERS>(p, g, C, keys, ids, n, HC, flag, s);
+    default: return launch_k1r<IDS>(p, g, C, keys, ids, n, HC, flag, s);
+  }
+}
+
+bool use_ranged(const ms_plan_s *p, uint64_t L) {
+  return p->ranged == 2 || (p->ranged == 1 && L >= 8ull * (uint64_t)sm_count());
 }
 
 ms_status check_ws(const ms_plan_s *p, uint64_t n, void *ws, size_t ws_bytes, Geometry *g) {
@@ -229,8 +277,9 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   const uint32_t m = spec->m;
   if (m < 1 || m > (uint32_t)kMaxM) return MS_ERR_INVALID_ARG;
   if (max_n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
-  if ((flags & MS_VARIANT_3K) && (flags & MS_VARIANT_1P)) return MS_ERR_INVALID_ARG;
-  if (flags & ~(MS_VALIDATE | MS_VARIANT_3K | MS_VARIANT_1P)) return MS_ERR_INVALID_ARG;
+  if ((flags & MS_VARIANT_3K) && (flags & MS_VARIANT_RANGED)) return MS_ERR_INVALID_ARG;
+  if (flags & ~(MS_VALIDATE | MS_VARIANT_3K | MS_VARIANT_RANGED)) return MS_ERR_INVALID_ARG;
+  if ((flags & MS_VARIANT_RANGED) && m > 32) return MS_ERR_UNSUPPORTED;
   BucketParams bp;
   memset(&bp, 0, sizeof(bp));
   int kkind = spec->kind;
@@ -290,6 +339,22 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
   if (const char *e = getenv("MS_K3_REVERSE")) p->bp.reverse = atoi(e) ? 1u : 0u;
   if (const char *e = getenv("MS_K3_NT")) p->k3nt = atoi(e) == 128 ? 128u : 256u;
+  // variant: CTA ranges for m <= 32 when a tile's mean bucket
+  // run is >= 256 keys (1 KB).  With shorter runs the strided tile walk wins:
+  // its concurrently processed tiles write ADJACENT runs of every bucket (m
+  // dense write streams), while contiguous ranges scatter them over C*m
+  // streams.  Forced either way by MS_VARIANT_3K / MS_VARIANT_RANGED (and
+  // MS_VARIANT=tile|ranged in the environment, for A/B measurements).
+  // Small inputs (L < 8 tiles per SM) keep the tile variant: a range is then
+  // only one or two tiles and the per-range setup is pure overhead.
+  p->ranged = (m <= 32 && p->k3nt * p->kpt >= 256u * m) ? 1 : 0;
+  if (const char *e = getenv("MS_VARIANT")) {
+    if (strcmp(e, "tile") == 0) p->ranged = 0;
+    if (strcmp(e, "ranged") == 0 && m <= 32) p->ranged = 2;
+  }
+  if (flags & MS_VARIANT_3K) p->ranged = 0;
+  if (flags & MS_VARIANT_RANGED) p->ranged = 2;
+  if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   *plan = p;
   return MS_OK;
 }
@@ -313,7 +378,7 @@ ms_status ms_plan_geometry(ms_plan_t p, uint64_t n, uint32_t *tile, uint64_t *nu
   Geometry g = geometry(p, n);
   if (tile) *tile = g.T;
   if (num_tiles) *num_tiles = g.L;
-  if (variant) *variant = 0;
+  if (variant) *variant = use_ranged(p, g.L) ? 1 : 0;
   return MS_OK;
 }
 
@@ -322,7 +387,8 @@ int32_t ms_plan_last_launches(ms_plan_t p) { return p ? p->last_launches : -1; }
 ms_status ms_plan_trace(ms_plan_t p, int enable) {
   if (!p) return MS_ERR_INVALID_ARG;
   if (enable) p->trace_runs = 0;
-  p->tracing = enable ? 1 : 0;
+  p->tracing = enable == 2 ? 2 : (enable ? 1 : 0);
+  if (enable) p->trace_mode = p->tracing;
   return MS_OK;
 }
 
@@ -332,8 +398,11 @@ ms_status ms_plan_trace_read(ms_plan_t p, float *stage_ms, int32_t max_runs, int
   for (int32_t i = 0; i < r; ++i) {
     cudaEvent_t *ev = &p->trace_ev[4 * i];
     if (cudaEventSynchronize(ev[3]) != cudaSuccess) return MS_ERR_CUDA;
-    for (int s = 0; s < 3; ++s)
-      if (cudaEventElapsedTime(&stage_ms[4 * i + s], ev[s], ev[s + 1]) != cudaSuccess) return MS_ERR_CUDA;
+    for (int s = 0; s < 3; ++s) {
+      stage_ms[4 * i + s] = 0.f;  // whole-run mode (2): no per-stage events
+      if (p->trace_mode != 2 && cudaEventElapsedTime(&stage_ms[4 * i + s], ev[s], ev[s + 1]) != cudaSuccess)
+        return MS_ERR_CUDA;
+    }
     if (cudaEventElapsedTime(&stage_ms[4 * i + 3], ev[0], ev[3]) != cudaSuccess) return MS_ERR_CUDA;
   }
   if (runs) *runs = r;
@@ -428,14 +497,41 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
     return MS_ERR_CUDA;
   cudaEvent_t *ev = trace_next(p);
   if (ev) cudaEventRecord(ev[0], s);
+  // K2 and K3 use programmatic dependent launch unless per-stage events sit
+  // between the kernels (tracing == 1) or MS_PDL=0
+  const bool pdl = p->pdl && p->tracing != 1;
+  if (use_ranged(p, g.L)) {  // K1r -> K2r -> K3 over C contiguous tile ranges (ms_ranged.cuh)
+    uint32_t C = 0;
+    if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 1, &C) != cudaSuccess ||
+        C == 0)
+      return MS_ERR_CUDA;
+    uint32_t *HC = (uint32_t *)(w + g.off_hc), *GB = (uint32_t *)(w + g.off_gb);
+    if (dispatch_k1r(p, g, C, keys_in, ids, (uint32_t)n, HC, flag, s) != cudaSuccess) return MS_ERR_CUDA;
+    if (ev && p->tracing == 1) cudaEventRecord(ev[1], s);
+    const uint32_t ksub = k1r_split(C), R = C * ksub;
+    const size_t smem2 = (size_t)R * p->spec.m * 4;
+    set_smem(k2r_scan, smem2);
+    if (launch_ex(pdl, k2r_scan, dim3(1), dim3(kR2Threads), smem2, s, (const uint32_t *)HC, GB, R, ksub, p->spec.m,
+                  std::max<uint32_t>(1, ceil_log2(p->spec.m)), offsets, (uint32_t)n) != cudaSuccess ||
+        cudaGetLastError() != cudaSuccess)
+      return MS_ERR_CUDA;
+    if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
+    if (dispatch_k3(p, g, keys_in, vals_in, ids, GB, keys_out, vals_out, (uint32_t)n, s, 1, nullptr, pdl) !=
+        cudaSuccess)
+      return MS_ERR_CUDA;
+    if (ev) cudaEventRecord(ev[3], s);
+    p->last_launches = 3;
+    return MS_OK;
+  }
   cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, status, (uint32_t)g.chunks, flag, s);
   if (e != cudaSuccess) return MS_ERR_CUDA;
-  if (ev) cudaEventRecord(ev[1], s);
-  k2_scan<<<(unsigned)g.chunks, kThreads, 0, s>>>(HG, g.hg_words, status, offsets, (uint32_t)g.L,
-                                                 p->spec.m, (uint32_t)n);
-  if (cudaGetLastError() != cudaSuccess) return MS_ERR_CUDA;
-  if (ev) cudaEventRecord(ev[2], s);
-  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, s);
+  if (ev && p->tracing == 1) cudaEventRecord(ev[1], s);
+  if (launch_ex(pdl, k2_scan, dim3((unsigned)g.chunks), dim3(kThreads), 0, s, HG, (uint64_t)g.hg_words, status,
+                offsets, (uint32_t)g.L, p->spec.m, (uint32_t)n) != cudaSuccess ||
+      cudaGetLastError() != cudaSuccess)
+    return MS_ERR_CUDA;
+  if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
+  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, s, 0, nullptr, pdl);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev) cudaEventRecord(ev[3], s);
   p->last_launches = 3;

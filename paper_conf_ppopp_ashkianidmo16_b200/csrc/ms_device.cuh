@@ -90,6 +90,14 @@ __device__ __forceinline__ uint32_t load_id(const void *ids, uint64_t i, const B
 }
 
 // ------------------------------------------------------------------ PTX helpers
+// Programmatic dependent launch (sm_90+): a kernel launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization may start while its
+// predecessor in the stream is still running; pdl_wait() blocks until the
+// predecessor grid has completed and its memory is visible (a no-op without
+// the attribute); pdl_trigger() lets the successor's CTAs be scheduled.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }

@@ -127,11 +127,15 @@ __device__ __forceinline__ void k3p_prefetch(uint32_t *stk, uint32_t *stv, uint3
 }
 
 // One tile, already staged.  FULL: all T keys valid (no per-key predicates).
-template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, int NT, bool FULL>
+// RANGED (ms_ranged.cuh): G_j of this tile is the running sum `grun` held by
+// the threads of bucket row j (advanced here by the tile's row total) instead
+// of a column of the global G array.
+template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, int NT, bool FULL, bool RANGED>
 __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *sm_v, const uint32_t *sm_i,
                                          const void *__restrict__ ids, uint32_t *__restrict__ keys_out,
                                          uint32_t *__restrict__ vals_out, uint64_t base, uint32_t nt,
-                                         const BucketParams &p, uint32_t *sm, uint32_t beta, uint32_t *meta) {
+                                         const BucketParams &p, uint32_t *sm, uint32_t beta, uint32_t *meta,
+                                         uint32_t &grun) {
   using Ly = K3pLayout<LOGMP, KV, IDS8, KPT, NT>;
   constexpr int MP = Ly::MP, K = Ly::K, CH = Ly::CH;
   constexpr int NW = NT / 32;
@@ -276,7 +280,23 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   if (tid == 0) rowS[MP] = tot;
   // padded run start P_j = S_j + 3j + ((G_j - S_j - 3j) & 3): P_j = G_j (mod 4)
   // and P_j >= P_{j-1} + h_{j-1}; closed form, no serial dependency over j.
-  const uint32_t Gr = row < m ? Gj[row] : 0u;
+  uint32_t Gr;
+  if constexpr (RANGED) {
+    Gr = grun;
+    uint32_t rtot;  // this tile's count of bucket `row`
+    if constexpr (TPR < 32) {
+      rtot = __shfl_sync(0xFFFFFFFFu, excl + s, lane | (TPR - 1)) - Sr;
+    } else {
+      rtot = 0;
+      const uint32_t w0 = (row * TPR) >> 5;
+#pragma unroll
+      for (int i = 0; i < NW; ++i) rtot += ((uint32_t)i >= w0 && (uint32_t)i < w0 + TPR / 32) ? wsum[i] : 0u;
+    }
+    grun += rtot;
+    if ((tid & (TPR - 1)) == 0) Gj[row] = Gr;
+  } else {
+    Gr = row < m ? Gj[row] : 0u;
+  }
   const uint32_t pad = 3 * row + ((Gr - Sr - 3 * row) & 3u);
 #pragma unroll
   for (int i = 0; i < NC; ++i) {
@@ -379,7 +399,7 @@ __device__ __forceinline__ void k3p_tile(const uint32_t *sm_k, const uint32_t *s
   }
 }
 
-template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, int NT>
+template <int KIND, bool KV, int LOGMP, bool IDS8, int KPT, int NT, bool RANGED>
 __global__ void __launch_bounds__(NT, NT == 256 ? (KV ? 2 : 3) : (KV ? 4 : 6))
 k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const void *__restrict__ ids, const uint32_t *__restrict__ G,
@@ -387,6 +407,7 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
              uint32_t L, const __grid_constant__ BucketParams p) {
   using Ly = K3pLayout<LOGMP, KV, IDS8, KPT, NT>;
   constexpr int T = Ly::T, STAGES = Ly::STAGES, CW = Ly::CW, MP = Ly::MP, K = Ly::K;
+  constexpr int LOGNT = NT == 256 ? 8 : 7;
   extern __shared__ __align__(128) uint32_t sm[];
   uint32_t *stk = sm + Ly::O_STK;
   uint32_t *stv = sm + Ly::O_STV;
@@ -394,18 +415,24 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t beta = 2 * lane + (warp & 1) + 64 * (warp >> 1);
   const uint32_t m = p.m;
-  // tiles blockIdx.x, blockIdx.x + gridDim.x, ...; the partial tile (if any)
-  // is the last one overall, hence the last of its CTA: it is peeled off
-  // the loop so its predicated code does not raise the loop's registers.
-  // p.reverse: walk tiles last-to-first, so the first tiles K3 reads are the
-  // ones K1 read last (still in the 126 MB L2); the partial tile is then the
-  // FIRST tile of CTA 0 instead of the last of its CTA.
-  const bool rev = p.reverse != 0;
+  // Tile mode: tiles blockIdx.x, blockIdx.x + gridDim.x, ...; the partial
+  // tile (if any) is the last one overall, hence the last of its CTA: it is
+  // peeled off the loop so its predicated code does not raise the loop's
+  // registers.  p.reverse: walk tiles last-to-first, so the first tiles K3
+  // reads are the ones K1 read last (still in the 126 MB L2); the partial
+  // tile is then the FIRST tile of CTA 0 instead of the last of its CTA.
+  // RANGED: CTA c walks its contiguous range [c*L/C, (c+1)*L/C) in order
+  // (G = GB[c][:], the range's bucket starts; the partial tile, if any, is
+  // the last tile of the last range).
+  const bool rev = !RANGED && p.reverse != 0;
+  const uint64_t r0 = RANGED ? (uint64_t)blockIdx.x * L / gridDim.x : 0;
   auto tile_of = [&](uint32_t it) -> uint64_t {
+    if constexpr (RANGED) return r0 + it;
     const uint64_t t = (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x;
     return rev ? (uint64_t)L - 1 - t : t;
   };
-  const uint32_t iters = blockIdx.x < L ? (L - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  const uint32_t iters = RANGED ? (uint32_t)((uint64_t)(blockIdx.x + 1) * L / gridDim.x - r0)
+                                : (blockIdx.x < L ? (L - 1 - blockIdx.x) / gridDim.x + 1 : 0);
   const bool partial = (uint64_t)n < (uint64_t)L * T;
   const bool tail_first = partial && rev && iters && blockIdx.x == 0;
   const bool has_tail = partial && !rev && iters && tile_of(iters - 1) == L - 1;
@@ -420,8 +447,15 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     if ((uint32_t)s < iters) k3p_prefetch<KV, IDS8, T, K, NT>(stk, stv, sti, s, keys, vals, ids, tile_of(s), n, beta);
     cp_async_commit();
   }
-  uint32_t gnext = 0;
-  if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
+  pdl_wait();  // K2's G / GB is complete (the first tiles' loads above are already in flight)
+  uint32_t gnext = 0;  // tile mode: the next tile's G column
+  uint32_t grun = 0;   // RANGED: G_row of the current tile (all threads of bucket row `row`)
+  if constexpr (RANGED) {
+    const uint32_t row = tid >> (LOGNT - LOGMP);
+    if (iters && row < m) grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
+  } else {
+    if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
+  }
 
   // per-iteration prologue: zero the counters (last read by the previous
   // tile's scatter, before a barrier), publish G[:, tile] into this parity's
@@ -435,8 +469,10 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
         if (idx < CW / 4) c4[idx] = make_uint4(0, 0, 0, 0);
       }
     }
-    if (tid < m) meta[MP + 4 + MP + tid] = gnext;
-    if (it + 1 < iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(it + 1));
+    if constexpr (!RANGED) {
+      if (tid < m) meta[MP + 4 + MP + tid] = gnext;
+      if (it + 1 < iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(it + 1));
+    }
     cp_async_wait<STAGES - 1>();
     __syncthreads();
   };
@@ -446,8 +482,8 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const uint64_t tile = tile_of(0);
     uint32_t *meta = sm + Ly::O_META;
     begin_tile(0, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, false>(stk, stv, sti, ids, keys_out, vals_out, tile * T,
-                                                (uint32_t)(n - tile * T), p, sm, beta, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, false, RANGED>(stk, stv, sti, ids, keys_out, vals_out, tile * T,
+                                                (uint32_t)(n - tile * T), p, sm, beta, meta, grun);
     if (STAGES < iters) k3p_prefetch<KV, IDS8, T, K, NT>(stk, stv, sti, 0, keys, vals, ids, tile_of(STAGES), n, beta);
     cp_async_commit();
     it = 1;
@@ -457,8 +493,8 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const int st = (int)(it % STAGES);
     uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
     begin_tile(it, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, true>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
-                                               vals_out, tile * T, T, p, sm, beta, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, true, RANGED>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids,
+                                                       keys_out, vals_out, tile * T, T, p, sm, beta, meta, grun);
     // refill this stage with tile it + STAGES (own chunks only; already consumed)
     if (it + STAGES < iters)
       k3p_prefetch<KV, IDS8, T, K, NT>(stk, stv, sti, st, keys, vals, ids, tile_of(it + STAGES), n, beta);
@@ -469,8 +505,9 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
     const int st = (int)(it % STAGES);
     uint32_t *meta = sm + Ly::O_META + (it & 1) * Ly::MW;
     begin_tile(it, meta);
-    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, false>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids, keys_out,
-                                                vals_out, tile * T, (uint32_t)(n - tile * T), p, sm, beta, meta);
+    k3p_tile<KIND, KV, LOGMP, IDS8, KPT, NT, false, RANGED>(stk + st * T, stv + st * T, sti + st * Ly::IW, ids,
+                                                        keys_out, vals_out, tile * T, (uint32_t)(n - tile * T), p,
+                                                        sm, beta, meta, grun);
   }
   bulk_wait_read0();
 }
@@ -483,20 +520,32 @@ inline cudaError_t k3p_launch_one(Kern k, size_t smem, const K3pArgs &a) {
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, NT, smem);
   if (per_sm <= 0) per_sm = 1;
   if (a.bp->dbg >= 10 && (int)(a.bp->dbg - 10) < per_sm) per_sm = (int)(a.bp->dbg - 10);  // ablation: CTAs/SM
-  const unsigned grid = (unsigned)umin64_host(a.L, (uint64_t)a.sms * per_sm);
-  k<<<grid, NT, smem, a.stream>>>(a.keys, a.vals, a.ids, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
-  return cudaGetLastError();
+  uint64_t g = umin64_host(a.L, (uint64_t)a.sms * per_sm);
+  if (a.ranged) g = umin64_host(g, kMaxRanges);
+  const unsigned grid = (unsigned)g;
+  if (a.grid_out) {
+    *a.grid_out = grid;
+    return cudaSuccess;
+  }
+  const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, a.keys, a.vals, a.ids, a.G,
+                                  a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+  return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+template <int KIND, bool KV, int LOGMP, int KPT, int NT, bool RANGED>
+inline cudaError_t k3p_launch_r(const K3pArgs &a) {
+  if constexpr (KIND == IDS) {
+    if (a.id_bytes == 1)
+      return k3p_launch_one<NT>(k3p_postscan<KIND, KV, LOGMP, true, KPT, NT, RANGED>,
+                                K3pLayout<LOGMP, KV, true, KPT, NT>::BYTES, a);
+  }
+  return k3p_launch_one<NT>(k3p_postscan<KIND, KV, LOGMP, false, KPT, NT, RANGED>,
+                            K3pLayout<LOGMP, KV, false, KPT, NT>::BYTES, a);
 }
 
 template <int KIND, bool KV, int LOGMP, int KPT, int NT>
 inline cudaError_t k3p_launch_n(const K3pArgs &a) {
-  if constexpr (KIND == IDS) {
-    if (a.id_bytes == 1)
-      return k3p_launch_one<NT>(k3p_postscan<KIND, KV, LOGMP, true, KPT, NT>,
-                                K3pLayout<LOGMP, KV, true, KPT, NT>::BYTES, a);
-  }
-  return k3p_launch_one<NT>(k3p_postscan<KIND, KV, LOGMP, false, KPT, NT>,
-                            K3pLayout<LOGMP, KV, false, KPT, NT>::BYTES, a);
+  return a.ranged ? k3p_launch_r<KIND, KV, LOGMP, KPT, NT, true>(a) : k3p_launch_r<KIND, KV, LOGMP, KPT, NT, false>(a);
 }
 
 template <int KIND, bool KV, int LOGMP, int KPT>

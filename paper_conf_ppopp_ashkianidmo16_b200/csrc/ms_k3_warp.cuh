@@ -176,6 +176,7 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   }
   // per-bucket setup while the copy is in flight
   uint32_t gcol = 0;
+  pdl_wait();  // K2's G is complete (the tile's TMA load above is already in flight)
   if (tid < m) gcol = __ldg(G + (uint64_t)tid * L + tile);
 #pragma unroll
   for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] = 0;  // kThreads == kMaxM
@@ -205,8 +206,9 @@ inline cudaError_t k3w_launch_l(const K3pArgs &a) {
   auto k = k3_postscan<KIND, KV, R, LOGM>;
   const size_t smem = k3w_smem(R, KV, id8);
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k<<<a.L, kThreads, smem, a.stream>>>(a.keys, a.vals, a.ids, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
-  return cudaGetLastError();
+  const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(a.L), dim3(kThreads), smem, a.stream, a.keys, a.vals, a.ids,
+                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 template <int KIND, bool KV, int R>

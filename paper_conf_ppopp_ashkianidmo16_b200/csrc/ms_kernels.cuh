@@ -54,6 +54,7 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
 #pragma unroll
     for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * NTS + tl);  // coalesced 128-bit loads
   }
+  pdl_trigger();  // K2 (launched with PDL) may be scheduled once every K1 CTA has started
   // K2's look-back status words are cleared here (K1 precedes K2 in the stream).
   for (uint32_t i = blockIdx.x * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
   uint4 *c4 = reinterpret_cast<uint4 *>(c8);
@@ -152,6 +153,8 @@ k2_scan(uint32_t *__restrict__ data, uint64_t total, uint64_t *__restrict__ stat
   const uint64_t chunk = blockIdx.x;
   const uint64_t base = chunk * kScanChunk;
   const uint32_t cnt = (uint32_t)umin64(kScanChunk, total - base);
+  pdl_wait();     // K1's H and zeroed status words are complete and visible
+  pdl_trigger();
 
 #pragma unroll
   for (int j = 0; j < kScanItems; ++j) {

@@ -50,16 +50,48 @@ NS = [0, 1, 31, 2047, 2048, 2049, 4095, 4097, 8191, 8193, 100003]
 MS = [1, 2, 3, 5, 8, 31, 32, 33, 64, 127, 255, 256]
 
 
+@pytest.mark.parametrize("variant", [None, "ranged"])
 @pytest.mark.parametrize("kind", ["lowbits", "delta", "splitters", "ids"])
 @pytest.mark.parametrize("m", MS)
-def test_parity_matrix(kind, m):
-    """kind x m x n (empty, ragged, tile edges) x KO/KV, uniform keys."""
+def test_parity_matrix(kind, m, variant):
+    """kind x m x n (empty, ragged, tile edges) x KO/KV, uniform keys; the default
+    variant (tile at these sizes) and the forced CTA-range variant (m <= 32)."""
     if kind == "lowbits" and m & (m - 1):
         pytest.skip("low-bit buckets need a power-of-two m (reading #10)")
+    if variant == "ranged" and m > 32:
+        pytest.skip("m > 32 always uses the tile variant")
     for i, n in enumerate(NS):
         for kv in (False, True):
             case = make_case(kind, m, n, seed=1000 * m + i, kv=kv, id_bytes=1 if i % 2 else 4)
-            _assert_equal(case, _run_case(case), _expect(case), f"{kind} m={m} n={n} kv={kv}")
+            _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} n={n} kv={kv} {variant}")
+
+
+@pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("ids", 5, True),
+                                       ("lowbits", 2, False), ("delta", 32, True)])
+def test_ranged_range_edges(kind, m, kv):
+    """Ranged variant around C = resident K3 CTAs: L < C, L = C +- 1, L = 3C + r (ranges of 1..4 tiles,
+    the ragged last tile at the end of the last range)."""
+    P = _pkg()
+    probe = P.Plan(P.BucketSpec(**make_case(kind, m, 1, 0, kv=kv)["spec_kw"]), 1 << 24, with_values=kv,
+                   variant="ranged")
+    T, _, v = probe.geometry(1 << 24)
+    assert v == 1
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    for i, L in enumerate([sms - 1, 2 * sms, 4 * sms + 1, 6 * sms - 1, 6 * sms, 6 * sms + 1, 13 * sms + 7]):
+        for n in (L * T, L * T - T + 3):
+            case = make_case(kind, m, n, seed=77 + i, kv=kv)
+            _assert_equal(case, _run_case(case, "ranged"), _expect(case), f"{kind} m={m} L={L} n={n}")
+
+
+@pytest.mark.parametrize("kv", [False, True])
+def test_parity_2p28_m32(kv):
+    """Headline size n = 2^28, m = 32 (DELTA 2^27, the NS configs), full element-wise compare."""
+    n = 1 << 28
+    keys = W.keys_np(n, W.SEEDS["C4"])
+    vals = W.values_np(n, W.SEEDS["C4"], "random") if kv else None
+    case = dict(spec_kw=dict(kind="delta", m=32, delta=1 << 27), ospec=oracle.Spec("delta", 32, delta=1 << 27),
+                keys=keys, vals=vals, ids=None)
+    _assert_equal(case, _run_case(case), _expect(case), "2^28 m=32")
 
 
 @pytest.mark.parametrize("dist", ["buckets", "binomial", "hot", "one"])
@@ -69,14 +101,17 @@ def test_parity_distributions(kind, m, dist):
     """Skewed workloads (§6.5): binomial, 75 % hot bucket, all in one bucket."""
     for n in (4097, (1 << 20) + 7):
         case = make_case(kind, m, n, seed=7 + m, dist=dist, kv=True)
-        _assert_equal(case, _run_case(case), _expect(case), f"{kind} m={m} {dist} n={n}")
+        for variant in ([None, "ranged"] if m <= 32 else [None]):
+            _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} {dist} n={n} {variant}")
 
 
-@pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("lowbits", 32, True)])
-def test_parity_2p25(kind, m, kv):
-    """BJ configs C2 / C3 size (n = 2^25), full element-wise compare."""
+@pytest.mark.parametrize("variant", [None, "3k", "ranged"])
+@pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("lowbits", 32, True),
+                                       ("lowbits", 2, True)])
+def test_parity_2p25(kind, m, kv, variant):
+    """BJ configs C2 / C3 size (n = 2^25), full element-wise compare, every variant."""
     case = make_case(kind, m, 1 << 25, seed=W.SEEDS["C3"], kv=kv, vals_kind="random")
-    _assert_equal(case, _run_case(case), _expect(case), f"2^25 {kind} m={m}")
+    _assert_equal(case, _run_case(case, variant), _expect(case), f"2^25 {kind} m={m} {variant}")
 
 
 @pytest.mark.parametrize("kv", [False, True])
