@@ -31,6 +31,7 @@ struct ms_plan_s {
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt (MS_K3_NT)
   int ranged = 0;  // CTA-range variant (ms_ranged.cuh, m <= 32): 0 never, 1 when L is large, 2 always
   int pdl = 1;     // programmatic dependent launch of K2, K3 (MS_PDL=0 disables)
+  int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
   int tracing = 0;     // 0 off, 1 per-stage events, 2 whole-run events only
@@ -183,6 +184,15 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   a.ranged = ranged;
   a.grid_out = grid_out;
   a.pdl = pdl;
+  if (p->spec.m <= 32 && p->k3v && p->kkind != IDS) {  // K3 v2 (ms_k3_v2.cuh)
+    switch (p->kkind) {
+      case LOWBITS: return k3v_launch_lowbits(a);
+      case SHIFTC: return k3v_launch_shiftc(a);
+      case SHIFT: return k3v_launch_shift(a);
+      case DELTA: return k3v_launch_delta(a);
+      default: return k3v_launch_splitters(a);
+    }
+  }
   if (p->spec.m <= 32) {  // persistent blocked-rank K3 (ms_k3_blocked.cuh), one TU per kind
     switch (p->kkind) {
       case LOWBITS: return k3p_launch_lowbits(a);
@@ -355,6 +365,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (flags & MS_VARIANT_3K) p->ranged = 0;
   if (flags & MS_VARIANT_RANGED) p->ranged = 2;
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
+  if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
   *plan = p;
   return MS_OK;
 }

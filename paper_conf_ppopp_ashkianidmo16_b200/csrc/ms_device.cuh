@@ -69,6 +69,43 @@ __device__ __forceinline__ uint32_t id_splitters(uint32_t k, const uint32_t *S, 
   return pos;
 }
 
+// ---- SPLITTERS through a bin table (DESIGN.md §7 "splitter bin table").
+// The key domain is cut into 1024 bins of W = 2^22 keys.  For bin b
+// (keys [b*W, (b+1)*W)) let lo = #{j : s_j < b*W} and c = the number of
+// splitters in [b*W, b*W + W - 2] (a splitter equal to the bin's last key is
+// never < a key of the bin).  Then for k in bin b, #{j : s_j < k} =
+//   c == 0: lo;   c == 1: lo + ((k - b*W) > (s_lo - b*W));   c >= 2: lo + #{...}
+// Entry: bit 31 = (c >= 2), bits 23..30 = lo, bits 0..22 = s_lo - b*W when
+// c == 1, else 0x7FFFFF (larger than any in-bin offset: the compare is false).
+// The c >= 2 case (rare for random splitters) walks the splitters from lo.
+constexpr int kSplBins = 1024;
+constexpr uint32_t kSplBinShift = 22;
+constexpr uint32_t kSplOffMask = (1u << kSplBinShift) - 1;
+
+__device__ __forceinline__ uint32_t id_spl_table(uint32_t k, const uint32_t *tbl, const uint32_t *S) {
+  const uint32_t e = tbl[k >> kSplBinShift];
+  uint32_t id = ((e >> 23) & 0xFFu) + ((k & kSplOffMask) > (e & 0x7FFFFFu) ? 1u : 0u);
+  if ((int32_t)e < 0) {
+    while (S[id] < k) ++id;  // S is padded with 0xFFFFFFFF: the walk stops by id = m - 1
+  }
+  return id;
+}
+
+// Build the bin table in shared memory from the padded splitters S (already
+// in shared memory); NT threads, each computes kSplBins / NT entries with two
+// branchless searches (lo and lo + c).
+template <int NT>
+__device__ __forceinline__ void build_spl_table(uint32_t *tbl, const uint32_t *S, uint32_t logm) {
+  for (uint32_t b = threadIdx.x; b < (uint32_t)kSplBins; b += NT) {
+    const uint32_t bs = b << kSplBinShift;
+    const uint32_t lo = id_splitters(bs, S, logm);
+    const uint32_t hi = id_splitters(bs + kSplOffMask, S, logm);  // #{s_j < bs + W - 1}
+    const uint32_t c = hi - lo;
+    tbl[b] = c == 0 ? (lo << 23) | 0x7FFFFFu
+                    : c == 1 ? (lo << 23) | (S[lo] - bs) : 0x80000000u | (lo << 23) | 0x7FFFFFu;
+  }
+}
+
 template <int KIND>
 __device__ __forceinline__ uint32_t bucket_of_key(uint32_t k, const BucketParams &p,
                                                   const uint32_t *spl_s) {
@@ -158,6 +195,20 @@ __device__ __forceinline__ void bulk_wait_read0() {
   asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// shared-memory accesses by 32-bit shared-window address (one IMAD/LEA per
+// address, in program order: the counting read-modify-write depends on it)
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+  uint16_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_u16(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((uint16_t)v) : "memory");
+}
+__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 inline uint64_t umin64_host(uint64_t a, uint64_t b) { return a < b ? a : b; }

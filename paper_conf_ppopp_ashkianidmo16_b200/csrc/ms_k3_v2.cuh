@@ -1,0 +1,496 @@
+// ms_k3_v2.cuh -- K3 post-scan for m <= 32, second generation (sm_100a).
+//
+// Same contract and the same paper steps as k3p_postscan (ms_k3_blocked.cuh):
+// recompute ids (footnote 6), stable local offsets (term 3 of
+// Eq. (2)) by an explicit, hierarchical H-bar scan,
+// a local stable multisplit of the tile in shared memory (§4 reordering,
+// P:689-713; §5.2.2), bucket runs written to G[j][tile] +
+// (slot - S_t[j]).  What changes is how the SM spends its instructions and
+// shared-memory wavefronts ("K3 v2"):
+//  * tiles are staged by the TMA engine (cp.async.bulk.tensor.2d, one
+//    instruction per array per tile, issued by one thread) with the 128-byte
+//    swizzle, so every thread reads its contiguous 16-key block as four
+//    conflict-free 128-bit loads with no address arithmetic per chunk;
+//  * keys stay in registers from the counting pass to the scatter; the key
+//    stage is handed back to the TMA right after counting, the value stage
+//    (key-value) after the scatter -- separate mbarriers per array;
+//  * the counter matrix is padded (16 B per 128 B) so that both the counting
+//    and the 128-bit scan accesses are conflict-free with no per-lane
+//    rotation, and the scan uses packed u16 arithmetic (3 instructions per
+//    2 counters: IMAD, IMAD, IDP2A);
+//  * counters and reordered keys are addressed by 32-bit shared-window
+//    addresses (one IMAD per access);
+//  * splitter ids come from a 1024-bin table in shared memory (one load and
+//    a compare per key, ms_device.cuh id_spl_table).
+// Tile walk: tile mode (tiles blockIdx.x, blockIdx.x + gridDim.x, ..., G from
+// the global G column) or RANGED (contiguous range per CTA, running G, see
+// ms_ranged.cuh).  The partial last tile (if any) is loaded with predicated
+// plain loads straight into registers.
+#pragma once
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <type_traits>
+
+#include "ms_k3p_args.h"
+
+namespace ms {
+
+template <int LOGMP, bool KV, int NT, int STAGES>
+struct K3vLayout {
+  static constexpr int MP = 1 << LOGMP;         // bucket rows (m rounded up to a power of 2, >= 2)
+  static constexpr int K = 16;                  // keys per thread (one contiguous block)
+  static constexpr int T = NT * K;              // keys per tile
+  static constexpr int TB = T * 4;              // bytes of one staged array (keys or values)
+  static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // reorder slots incl. alignment padding
+  static constexpr int MW = 3 * MP + 8;         // per-tile metadata words: rowS[MP+4] P[MP] G[MP]
+  // u16 counter matrix c[j][beta], row-major, with 16 bytes of padding after
+  // every 128 bytes: byte o of the plain layout lives at o + 16 * (o / 128).
+  // Counting (32 lanes, 32 consecutive words of one row) and the scan
+  // (thread t reads the 4*WPT-byte segment t with 128-bit loads) are then
+  // both free of bank conflicts, without rotating any register order.
+  static constexpr int RS = 2 * NT + 2 * NT / 8;  // padded row stride (bytes)
+  static constexpr int CNTB = MP * RS;
+  // byte offsets from the 1024-byte-aligned base (128B swizzle needs 1024 B alignment)
+  static constexpr int O_SK = 0;                          // [STAGES][T] staged keys
+  static constexpr int O_SV = O_SK + STAGES * TB;         // [STAGES][T] staged values
+  static constexpr int O_KS = O_SV + (KV ? STAGES * TB : 0);  // reordered keys
+  static constexpr int O_VS = O_KS + KSR * 4;             // reordered values
+  static constexpr int O_CNT = O_VS + (KV ? KSR * 4 : 0); // counters
+  static constexpr int O_META = O_CNT + CNTB;             // [2][MW] words (tile parity)
+  static constexpr int O_WS = O_META + 2 * MW * 4;        // warp sums [16]
+  static constexpr int O_BAR = (O_WS + 16 * 4 + 7) & ~7;  // mbarriers: keys [STAGES], values [STAGES]
+  static constexpr int O_SPL = O_BAR + 2 * STAGES * 8;    // SPLITTERS: padded splitters [256] + bin table
+  static constexpr int O_TBL = O_SPL + kMaxM * 4;
+  static constexpr int BYTES = O_SPL;                     // + 1024 alignment slack at launch
+  static constexpr int BYTES_SPL = O_TBL + kSplBins * 4;
+};
+
+// TMA 2-D tensor load (box = T/32 rows of 32 keys) into shared memory, completion on `bar`.
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *tm, int c0, int c1, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(tm), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
+}
+
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB>
+__global__ void __launch_bounds__(NT, MINB)
+k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv,
+             const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
+             const uint32_t *__restrict__ G, uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
+             uint32_t n, uint32_t L, const __grid_constant__ BucketParams p) {
+  using Ly = K3vLayout<LOGMP, KV, NT, STAGES>;
+  constexpr int MP = Ly::MP, K = Ly::K, T = Ly::T, TB = Ly::TB, RS = Ly::RS;
+  constexpr int NW = NT / 32;
+  constexpr int LOGNT = NT == 256 ? 8 : 7;
+  constexpr bool KEEP_ID = KIND == SPLITTERS;  // the table lookup is kept, not repeated
+  extern __shared__ uint8_t smraw[];
+  // align to 1024 B by offsetting the shared pointer itself (an integer round
+  // trip would turn every access below into a generic LD/ST)
+  uint8_t *sm = smraw + ((1024u - (smem_u32(smraw) & 1023u)) & 1023u);
+  uint32_t *keys_s = reinterpret_cast<uint32_t *>(sm + Ly::O_KS);
+  uint32_t *vals_s = reinterpret_cast<uint32_t *>(sm + Ly::O_VS);
+  uint8_t *cnt = sm + Ly::O_CNT;
+  uint32_t *wsum = reinterpret_cast<uint32_t *>(sm + Ly::O_WS);
+  uint64_t *bar_k = reinterpret_cast<uint64_t *>(sm + Ly::O_BAR);
+  uint64_t *bar_v = bar_k + STAGES;
+  uint32_t *spl_s = reinterpret_cast<uint32_t *>(sm + Ly::O_SPL);
+  uint32_t *tbl_s = reinterpret_cast<uint32_t *>(sm + Ly::O_TBL);
+
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // block beta of this thread: the 32 lanes of a warp own 32 consecutive
+  // counter words of a row (32 banks) whatever their ids; the staged block is
+  // row beta >> 1, half beta & 1 of the swizzled 128-byte rows
+  const uint32_t beta = 2 * lane + (warp & 1) + 64 * (warp >> 1);
+  const uint32_t srow = beta >> 1, shalf = beta & 1;
+  uint32_t choff[4];  // byte offsets of the block's 4 chunks inside a stage (128B swizzle)
+#pragma unroll
+  for (int c = 0; c < 4; ++c) choff[c] = srow * 128 + 16 * ((4 * shalf + c) ^ (srow & 7));
+  const uint32_t m = p.m;
+  const uint32_t b0 = beta * K;
+  // c[j][beta] at shared address ccol + j * RS
+  const uint32_t ccol = smem_u32(cnt) + 2 * beta + 16 * (beta >> 6);
+  const uint32_t ks32 = smem_u32(keys_s), vs32 = smem_u32(vals_s);
+
+  const uint64_t r0 = RANGED ? (uint64_t)blockIdx.x * L / gridDim.x : 0;
+  auto tile_of = [&](uint32_t it) -> uint64_t {
+    return RANGED ? r0 + it : (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x;
+  };
+  const uint32_t iters = RANGED ? (uint32_t)((uint64_t)(blockIdx.x + 1) * L / gridDim.x - r0)
+                                : (blockIdx.x < L ? (L - 1 - blockIdx.x) / gridDim.x + 1 : 0);
+  const uint64_t Lfull = n / T;  // tiles the TMA loads; a partial last tile is loaded by hand
+  auto issue = [&](uint32_t it, bool values) {  // one thread: TMA of tile `it` into its stage
+    const uint64_t tile = tile_of(it);
+    if (tile >= Lfull) return;
+    const int st = (int)(it % STAGES);
+    if (!values) {
+      mbar_arrive_expect_tx(bar_k + st, TB);
+      tma_load_2d(sm + Ly::O_SK + st * TB, &tmk, 0, (int)(tile * (T / 32)), bar_k + st);
+    } else {
+      mbar_arrive_expect_tx(bar_v + st, TB);
+      tma_load_2d(sm + Ly::O_SV + st * TB, &tmv, 0, (int)(tile * (T / 32)), bar_v + st);
+    }
+  };
+
+  if (tid == 0) {
+#pragma unroll
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(bar_k + s, 1);
+      mbar_init(bar_v + s, 1);
+    }
+    fence_mbar_init();
+    for (uint32_t s = 0; s < (uint32_t)STAGES && s < iters; ++s) {
+      issue(s, false);
+      if constexpr (KV) issue(s, true);
+    }
+  }
+  if constexpr (KIND == SPLITTERS) {
+    for (uint32_t i = tid; i < (1u << p.logm); i += NT) spl_s[i] = p.spl[i];
+    __syncthreads();
+    build_spl_table<NT>(tbl_s, spl_s, p.logm);
+  }
+  auto id_of = [&](uint32_t key) -> uint32_t {
+    if constexpr (KIND == SPLITTERS) return id_spl_table(key, tbl_s, spl_s);
+    else return bucket_of_key<KIND>(key, p, spl_s);
+  };
+
+  pdl_wait();  // K2's G / GB is complete (the first tiles' loads above are already in flight)
+  uint32_t gnext = 0;  // tile mode: the next tile's G column
+  uint32_t grun = 0;   // RANGED: G_row of the current tile (all threads of bucket row `row`)
+  const uint32_t row = tid >> (LOGNT - LOGMP);
+  if constexpr (RANGED) {
+    if (iters && row < m) grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
+  } else {
+    if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
+  }
+
+  // one tile; FULL (compile time): all T keys valid, TMA-staged.  The partial
+  // tile (at most one, the last of its CTA) is peeled off the loop
+  auto tile_body = [&](uint32_t it, auto fullc) {
+    constexpr bool FULL = decltype(fullc)::value;
+    const uint64_t tile = tile_of(it);
+    const uint64_t base = tile * T;
+    const uint32_t nt = FULL ? (uint32_t)T : (uint32_t)(n - base);
+    const int st = (int)(it % STAGES);
+    const uint32_t ph = (it / STAGES) & 1u;
+    uint32_t *meta = reinterpret_cast<uint32_t *>(sm + Ly::O_META) + (it & 1) * Ly::MW;
+    uint32_t *rowS = meta;          // [MP+4]
+    uint32_t *Pj = meta + MP + 4;   // [MP]
+    uint32_t *Gj = Pj + MP;         // [MP]
+
+    // ---- 0. zero the counters (last read by the previous tile's scatter,
+    // before its final barrier); publish this tile's G column
+    {
+      uint4 *c4 = reinterpret_cast<uint4 *>(cnt);
+#pragma unroll
+      for (int i = 0; i < (Ly::CNTB / 16 + NT - 1) / NT; ++i) {
+        const int idx = i * NT + tid;
+        if (idx < Ly::CNTB / 16) c4[idx] = make_uint4(0, 0, 0, 0);
+      }
+    }
+    if constexpr (!RANGED) {
+      if (tid < m) Gj[tid] = gnext;
+      if (it + 1 < iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(it + 1));
+    }
+    __syncthreads();
+
+    // ---- 1. this thread's block -> registers; sequential counting into the
+    // private counter column (the value read is the key's rank in the block)
+    uint4 kx[4];
+    if constexpr (FULL) {
+      mbar_wait(bar_k + st, ph);
+      const uint8_t *sk = sm + Ly::O_SK + st * TB;
+#pragma unroll
+      for (int c = 0; c < 4; ++c) kx[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
+    } else {
+      uint32_t t[K];
+#pragma unroll
+      for (int q = 0; q < K; ++q) t[q] = b0 + q < nt ? __ldg(keys + base + b0 + q) : 0u;
+#pragma unroll
+      for (int c = 0; c < 4; ++c) kx[c] = make_uint4(t[4 * c], t[4 * c + 1], t[4 * c + 2], t[4 * c + 3]);
+    }
+    uint32_t rk[4];                     // ranks (< 16), one byte each
+    uint32_t idk[KEEP_ID ? 4 : 1];      // kept ids, one byte each
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
+      rk[c] = 0u;
+      if constexpr (KEEP_ID) idk[c] = 0u;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        if (FULL || b0 + 4 * c + j < nt) {
+          const uint32_t id = id_of(kk[j]);
+          const uint32_t a = ccol + id * RS;
+          const uint32_t r = lds_u16(a);
+          sts_u16(a, r + 1);
+          rk[c] |= r << (8 * j);
+          if constexpr (KEEP_ID) idk[c] |= id << (8 * j);
+        }
+      }
+    }
+    __syncthreads();
+    // the key stage is free again (keys are in registers): refill it
+    if (tid == 0 && it + STAGES < iters) issue(it + STAGES, false);
+
+    // ---- 2. CTA exclusive scan of the row-vectorised counter matrix:
+    // thread t owns plain words [t*WPT, (t+1)*WPT) (inside one bucket row)
+    constexpr int WPT = MP / 2;
+    constexpr int NC = WPT >= 4 ? WPT / 4 : 1;
+    constexpr int CWD = WPT >= 4 ? 4 : WPT;
+    uint8_t *seg = cnt + 4 * WPT * tid + 16 * ((4 * WPT * tid) >> 7);
+    uint32_t w[NC][CWD];
+    uint32_t s = 0;
+#pragma unroll
+    for (int i = 0; i < NC; ++i) {
+      const uint8_t *src = seg + 16 * i;
+      if constexpr (CWD == 4) {
+        const uint4 x = *reinterpret_cast<const uint4 *>(src);
+        w[i][0] = x.x; w[i][1] = x.y; w[i][2] = x.z; w[i][3] = x.w;
+      } else if constexpr (CWD == 2) {
+        const uint2 x = *reinterpret_cast<const uint2 *>(src);
+        w[i][0] = x.x; w[i][1] = x.y;
+      } else {
+        w[i][0] = *reinterpret_cast<const uint32_t *>(src);
+      }
+#pragma unroll
+      for (int j = 0; j < CWD; ++j) s = __dp2a_lo(w[i][j], 0x0101u, s);  // += lo + hi
+    }
+    const uint32_t incl = warp_incl_scan(s, lane);
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    uint32_t wpre = 0, tot = 0;
+#pragma unroll
+    for (int i = 0; i < NW; ++i) {
+      const uint32_t x = wsum[i];
+      wpre += (i < (int)warp) ? x : 0u;
+      tot += x;
+    }
+    const uint32_t excl = wpre + incl - s;
+    constexpr uint32_t TPR = NT >> LOGMP;  // threads per bucket row
+    uint32_t Sr;                           // S_row = excl of the row's first thread
+    if constexpr (TPR < 32) {
+      Sr = __shfl_sync(0xFFFFFFFFu, excl, lane & ~(TPR - 1));
+    } else {
+      Sr = 0;
+      const uint32_t w0 = (row * TPR) >> 5;
+#pragma unroll
+      for (int i = 0; i < NW; ++i) Sr += ((uint32_t)i < w0) ? wsum[i] : 0u;
+    }
+    if ((tid & (TPR - 1)) == 0) rowS[row] = excl;
+    if (tid == 0) rowS[MP] = tot;
+    uint32_t Gr;
+    if constexpr (RANGED) {
+      Gr = grun;
+      uint32_t rtot;  // this tile's count of bucket `row`
+      if constexpr (TPR < 32) {
+        rtot = __shfl_sync(0xFFFFFFFFu, excl + s, lane | (TPR - 1)) - Sr;
+      } else {
+        rtot = 0;
+        const uint32_t w0 = (row * TPR) >> 5;
+#pragma unroll
+        for (int i = 0; i < NW; ++i) rtot += ((uint32_t)i >= w0 && (uint32_t)i < w0 + TPR / 32) ? wsum[i] : 0u;
+      }
+      grun += rtot;
+      if ((tid & (TPR - 1)) == 0) Gj[row] = Gr;
+    } else {
+      Gr = row < m ? Gj[row] : 0u;
+    }
+    // padded run start P_j = S_j + 3j + ((G_j - S_j - 3j) & 3): P_j = G_j (mod 4)
+    // and P_j >= P_{j-1} + h_{j-1}; closed form, no serial dependency over j
+    const uint32_t pad = 3 * row + ((Gr - Sr - 3 * row) & 3u);
+    uint32_t run = excl + pad;
+#pragma unroll
+    for (int i = 0; i < NC; ++i) {
+#pragma unroll
+      for (int j = 0; j < CWD; ++j) {
+        const uint32_t x = w[i][j];
+        w[i][j] = x * 0x10000u + run * 0x10001u;  // (run, run + lo)
+        run = __dp2a_lo(x, 0x0101u, run);         // run + lo + hi
+      }
+      uint8_t *dst = seg + 16 * i;
+      if constexpr (CWD == 4) *reinterpret_cast<uint4 *>(dst) = make_uint4(w[i][0], w[i][1], w[i][2], w[i][3]);
+      else if constexpr (CWD == 2) *reinterpret_cast<uint2 *>(dst) = make_uint2(w[i][0], w[i][1]);
+      else *reinterpret_cast<uint32_t *>(dst) = w[i][0];
+    }
+    if ((tid & (TPR - 1)) == 0) Pj[row] = Sr + pad;
+    bulk_wait_read0();  // this thread's bulk stores of the previous tile have read keys_s/vals_s
+    __syncthreads();
+
+    // ---- 3. local multisplit of the tile into shared memory
+    uint4 vy[KV ? 4 : 1];
+    if constexpr (KV) {
+      if constexpr (FULL) {
+        mbar_wait(bar_v + st, ph);
+        const uint8_t *sv = sm + Ly::O_SV + st * TB;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) vy[c] = *reinterpret_cast<const uint4 *>(sv + choff[c]);
+      } else {
+        uint32_t t[K];
+#pragma unroll
+        for (int q = 0; q < K; ++q) t[q] = b0 + q < nt ? __ldg(vals + base + b0 + q) : 0u;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) vy[c] = make_uint4(t[4 * c], t[4 * c + 1], t[4 * c + 2], t[4 * c + 3]);
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
+      uint32_t vv[4];
+      if constexpr (KV) {
+        vv[0] = vy[c].x; vv[1] = vy[c].y; vv[2] = vy[c].z; vv[3] = vy[c].w;
+      }
+      uint32_t sl[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        uint32_t id;
+        if constexpr (KEEP_ID) id = __byte_perm(idk[c], 0u, 0x4440u + j);
+        else id = id_of(kk[j]);
+        sl[j] = (FULL || b0 + 4 * c + j < nt) ? lds_u16(ccol + id * RS) : 0u;
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        if (FULL || b0 + 4 * c + j < nt) {
+          const uint32_t slot = sl[j] + __byte_perm(rk[c], 0u, 0x4440u + j);
+          sts_u32(ks32 + 4 * slot, kk[j]);
+          if constexpr (KV) sts_u32(vs32 + 4 * slot, vv[j]);
+        }
+      }
+    }
+    fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA (async proxy)
+    __syncthreads();
+    if constexpr (KV) {  // the value stage is free again: refill it
+      if (tid == 0 && it + STAGES < iters) issue(it + STAGES, true);
+    }
+
+    // ---- 4. bucket runs: SPB threads per bucket share its <= 3 head keys,
+    // <= 3 tail keys and the TMA bulk store(s) of the 16-byte-aligned body
+    {
+      constexpr uint32_t SPB = NT / 32;
+      const uint32_t b = tid / SPB, sub = tid % SPB;
+      if (b < m) {
+        const uint32_t len = rowS[b + 1] - rowS[b];
+        const uint32_t P = Pj[b], Gd = Gj[b];
+        const uint32_t head = min(len, (4u - (Gd & 3u)) & 3u);
+        const uint32_t body = (len - head) & ~3u;
+        if constexpr (SPB == 8) {
+          if (sub < 6) {
+            const uint32_t i = sub < 3 ? sub : head + body + (sub - 3);
+            if ((sub < 3 && sub < head) || (sub >= 3 && i < len)) {
+              keys_out[Gd + i] = keys_s[P + i];
+              if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+            }
+          } else if (body && (sub == 6 || KV)) {
+            if (sub == 6) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
+            else bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
+            bulk_commit();
+          }
+        } else {  // SPB == 4: head / tail / keys body / values body
+          if (sub < 2) {
+            const uint32_t i0 = sub == 0 ? 0u : head + body, i1 = sub == 0 ? head : len;
+            for (uint32_t i = i0; i < i1; ++i) {
+              keys_out[Gd + i] = keys_s[P + i];
+              if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+            }
+          } else if (body && (sub == 2 || KV)) {
+            if (sub == 2) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
+            else bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
+            bulk_commit();
+          }
+        }
+      }
+    }
+  };
+  const bool has_tail = iters && tile_of(iters - 1) >= Lfull;
+  const uint32_t iters_full = iters - (has_tail ? 1u : 0u);
+  for (uint32_t it = 0; it < iters_full; ++it) tile_body(it, std::true_type{});
+  if (has_tail) tile_body(iters_full, std::false_type{});
+  bulk_wait_read0();
+}
+
+// ------------------------------------------------------------------ host launcher
+inline PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  }
+  return fn;
+}
+
+// keys (or values) of the `full` tiles as a [rows][32] u32 tensor, box = T/32 rows, 128B swizzle
+inline bool make_tile_map(CUtensorMap *tm, const uint32_t *ptr, uint64_t rows, uint32_t T) {
+  memset(tm, 0, sizeof(*tm));
+  if (!ptr || rows == 0) return true;  // no full tile: the map is never used
+  auto enc = tensor_map_encoder();
+  if (!enc) return false;
+  const cuuint64_t dims[2] = {32, rows};
+  const cuuint64_t strides[1] = {128};
+  const cuuint32_t box[2] = {32, T / 32};
+  const cuuint32_t es[2] = {1, 1};
+  return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(ptr), dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED>
+inline cudaError_t k3v_launch_one(const K3pArgs &a) {
+  using Ly = K3vLayout<LOGMP, KV, NT, STAGES>;
+  constexpr int MINB = NT == 256 ? (KV ? 2 : 3) : (KV ? 4 : 6);
+  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB>;
+  const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
+  cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, NT, smem);
+  if (per_sm <= 0) per_sm = 1;
+  uint64_t g = umin64_host(a.L, (uint64_t)a.sms * per_sm);
+  if (a.ranged) g = umin64_host(g, kMaxRanges);
+  const unsigned grid = (unsigned)g;
+  if (a.grid_out) {
+    *a.grid_out = grid;
+    return cudaSuccess;
+  }
+  const uint64_t rows = (uint64_t)(a.n / Ly::T) * (Ly::T / 32);
+  CUtensorMap tmk, tmv;
+  if (!make_tile_map(&tmk, a.keys, rows, Ly::T) || !make_tile_map(&tmv, KV ? a.vals : nullptr, rows, Ly::T))
+    return cudaErrorInvalidValue;
+  const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals,
+                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+  return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+template <int KIND, bool KV, int LOGMP, int NT>
+inline cudaError_t k3v_launch_n(const K3pArgs &a) {
+  constexpr int STAGES = KV ? 1 : 2;
+  return a.ranged ? k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true>(a)
+                  : k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false>(a);
+}
+
+template <int KIND, bool KV, int LOGMP>
+inline cudaError_t k3v_launch_l(const K3pArgs &a) {
+  return a.nt == 128 ? k3v_launch_n<KIND, KV, LOGMP, 128>(a) : k3v_launch_n<KIND, KV, LOGMP, 256>(a);
+}
+
+template <int KIND, bool KV>
+inline cudaError_t k3v_launch_kv(const K3pArgs &a) {
+  uint32_t l = 1;
+  while ((1u << l) < a.m) ++l;
+  switch (l) {
+    case 1: return k3v_launch_l<KIND, KV, 1>(a);
+    case 2: return k3v_launch_l<KIND, KV, 2>(a);
+    case 3: return k3v_launch_l<KIND, KV, 3>(a);
+    case 4: return k3v_launch_l<KIND, KV, 4>(a);
+    default: return k3v_launch_l<KIND, KV, 5>(a);
+  }
+}
+
+template <int KIND>
+inline cudaError_t k3v_launch(const K3pArgs &a) {
+  return a.vals ? k3v_launch_kv<KIND, true>(a) : k3v_launch_kv<KIND, false>(a);
+}
+
+}  // namespace ms

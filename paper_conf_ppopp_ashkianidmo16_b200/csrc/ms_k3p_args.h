@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstring>
 #include <utility>
 
 #include "ms_device.cuh"
@@ -51,6 +52,12 @@ cudaError_t k3p_launch_shift(const K3pArgs &a);
 cudaError_t k3p_launch_delta(const K3pArgs &a);
 cudaError_t k3p_launch_splitters(const K3pArgs &a);
 cudaError_t k3p_launch_ids(const K3pArgs &a);
+// m <= 32, second generation (ms_k3_v2.cuh): TMA-tensor staging, keys in registers
+cudaError_t k3v_launch_lowbits(const K3pArgs &a);
+cudaError_t k3v_launch_shiftc(const K3pArgs &a);
+cudaError_t k3v_launch_shift(const K3pArgs &a);
+cudaError_t k3v_launch_delta(const K3pArgs &a);
+cudaError_t k3v_launch_splitters(const K3pArgs &a);
 // m > 32: warp-ballot K3 (ms_k3_warp.cuh); kpt carries the rounds per warp R (8 or 16)
 cudaError_t k3w_launch_lowbits(const K3pArgs &a);
 cudaError_t k3w_launch_shiftc(const K3pArgs &a);
