@@ -126,7 +126,20 @@ void set_smem(K kernel, size_t bytes) {
   if (bytes > 48 * 1024) cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
 }
 
-size_t k1_smem(uint32_t m) { return kMaxM * 4 + (size_t)m * kThreads; }
+int sm_count() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
+
+size_t k1_smem(uint32_t m, int kind) {
+  return kMaxM * 4 + (kind == SPLITTERS ? kSplBins * 4 : 0) + (size_t)m * kThreads;
+}
 
 
 // ---------------------------------------------------------------- dispatch
@@ -134,13 +147,17 @@ template <int KIND>
 cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const void *ids,
                       uint32_t n, uint32_t *H, uint64_t *zero_ptr, uint32_t zero_words,
                       uint32_t *flag, cudaStream_t s) {
-  size_t smem = k1_smem(p->spec.m);
-#define MS_K1(KPT, SUBT)                                                                    \
-  {                                                                                          \
-    auto k = k1_prescan<KIND, KPT, SUBT>;                                                    \
-    set_smem(k, smem);                                                                       \
-    k<<<(unsigned)((g.L + SUBT - 1) / SUBT), kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, \
-                                                                 zero_ptr, zero_words, flag);  \
+  const size_t smem = k1_smem(p->spec.m, KIND);
+  // one CTA per tile group; SPLITTERS: k1s_prescan on a persistent grid (8 CTAs
+  // per SM) so the bin table is built once per CTA
+#define MS_K1(KPT, SUBT)                                                                          \
+  {                                                                                                \
+    auto k = KIND == SPLITTERS ? k1s_prescan<KIND, KPT, SUBT> : k1_prescan<KIND, KPT, SUBT>;      \
+    set_smem(k, smem);                                                                             \
+    uint64_t grid = (g.L + SUBT - 1) / SUBT;                                                       \
+    if (KIND == SPLITTERS) grid = std::min<uint64_t>(grid, 8ull * (uint64_t)sm_count());           \
+    k<<<(unsigned)grid, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, zero_words, \
+                                             flag);                                                \
   }
   switch (g.R) {  // 16 keys per thread; T = 2048 tiles are counted two per CTA
     case 8: MS_K1(16, 2) break;
@@ -164,16 +181,6 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   }
 }
 
-int sm_count() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
-  }
-  return sms;
-}
 
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
@@ -344,6 +351,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   // K3 CTA size (m <= 32), measured per workload: 256 threads
   // (T = 4096) for m > 16 with one-instruction ids, 128 (T = 2048) otherwise
   p->k3nt = (m > 16 && (kkind == SHIFT || kkind == SHIFTC || kkind == LOWBITS)) ? 256u : 128u;
+  if (kkind != IDS) p->k3nt = 256u;  // K3 v2: 256 threads (T = 4096) measured best for every m <= 32
   // ablation overrides: MS_DEBUG_K3=1 drops K3's global stores;
   // MS_K3_REVERSE=1 walks K3's tiles last-to-first
   if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
@@ -542,7 +550,11 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
       cudaGetLastError() != cudaSuccess)
     return MS_ERR_CUDA;
   if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
-  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, s, 0, nullptr, pdl);
+  // K3 after the many-CTA K2 of the tile variant: PDL only for key-only runs
+  // (measured: an early-resident key-value K3 -- 2 CTAs with
+  // the whole register file per SM -- costs ~6 % at n = 2^28)
+  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, s, 0, nullptr,
+                  pdl && vals_in == nullptr);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev) cudaEventRecord(ev[3], s);
   p->last_launches = 3;

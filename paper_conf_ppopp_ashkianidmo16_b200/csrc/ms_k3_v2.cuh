@@ -44,12 +44,14 @@ struct K3vLayout {
   static constexpr int TB = T * 4;              // bytes of one staged array (keys or values)
   static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // reorder slots incl. alignment padding
   static constexpr int MW = 3 * MP + 8;         // per-tile metadata words: rowS[MP+4] P[MP] G[MP]
-  // u16 counter matrix c[j][beta], row-major, with 16 bytes of padding after
-  // every 128 bytes: byte o of the plain layout lives at o + 16 * (o / 128).
-  // Counting (32 lanes, 32 consecutive words of one row) and the scan
-  // (thread t reads the 4*WPT-byte segment t with 128-bit loads) are then
-  // both free of bank conflicts, without rotating any register order.
-  static constexpr int RS = 2 * NT + 2 * NT / 8;  // padded row stride (bytes)
+  // u16 counter matrix c[j][beta], row-major; inside a row, 16 bytes of
+  // padding after every 128 bytes (byte q of a plain row lives at
+  // q + 16 * (q / 128)), and the row stride is rounded up to a multiple of
+  // 128 bytes.  Counting (32 lanes, 32 consecutive words of their rows: bank =
+  // lane whatever the row) and the scan (thread t reads the 4*WPT-byte
+  // segment t with 128-bit loads) are then both free of bank conflicts,
+  // without rotating any register order.
+  static constexpr int RS = (2 * NT + 2 * NT / 8 + 127) / 128 * 128;  // padded row stride (bytes)
   static constexpr int CNTB = MP * RS;
   // byte offsets from the 1024-byte-aligned base (128B swizzle needs 1024 B alignment)
   static constexpr int O_SK = 0;                          // [STAGES][T] staged keys
@@ -239,7 +241,9 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     constexpr int WPT = MP / 2;
     constexpr int NC = WPT >= 4 ? WPT / 4 : 1;
     constexpr int CWD = WPT >= 4 ? 4 : WPT;
-    uint8_t *seg = cnt + 4 * WPT * tid + 16 * ((4 * WPT * tid) >> 7);
+    constexpr uint32_t SEGS = 2 * NT / (4 * WPT);  // segments per row
+    const uint32_t q = 4 * WPT * (tid % SEGS);     // plain byte offset inside row tid / SEGS
+    uint8_t *seg = cnt + (tid / SEGS) * RS + q + 16 * (q >> 7);
     uint32_t w[NC][CWD];
     uint32_t s = 0;
 #pragma unroll

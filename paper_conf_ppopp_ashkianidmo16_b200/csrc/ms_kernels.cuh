@@ -132,6 +132,133 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   }
 }
 
+// Persistent form of K1 for MS_SPLITTERS: the bin table (ms_device.cuh) is
+// built once per CTA, then the CTA walks tile groups with a stride of gridDim.x.
+template <int KIND, int KPT, int SUBT>
+__global__ void __launch_bounds__(kThreads)
+k1s_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
+           uint32_t L, uint32_t *__restrict__ H, const __grid_constant__ BucketParams p,
+           uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
+  // SUBT tiles per CTA iteration: warps [h*8/SUBT, (h+1)*8/SUBT) count tile SUBT*group + h.
+  // The byte-counter slot layout puts warps 0-3 in bytes [0,128) of every row and
+  // warps 4-7 in [128,256), so each half-row is one tile's column.  CTAs walk
+  // the tile groups with a stride of gridDim.x (one group per CTA unless the
+  // launcher makes the grid persistent -- SPLITTERS, whose bin table is built
+  // once per CTA).
+  constexpr int NTS = kThreads / SUBT;   // threads per tile
+  constexpr int T = NTS * KPT;           // keys per tile
+  static_assert(KPT <= 255 && KPT % 4 == 0, "byte counters");
+  extern __shared__ __align__(16) uint32_t smem[];
+  uint32_t *spl_s = smem;                                     // kMaxM words (SPLITTERS)
+  uint32_t *tbl_s = smem + kMaxM;                             // kSplBins words (SPLITTERS)
+  uint8_t *c8 = reinterpret_cast<uint8_t *>(smem + kMaxM + (KIND == SPLITTERS ? kSplBins : 0));  // [m][256]
+  const uint32_t tid = threadIdx.x, lane = tid & 31;
+  const uint32_t h = tid / NTS, tl = tid % NTS;
+  const uint32_t m = p.m;
+  const uint64_t groups = ((uint64_t)L + SUBT - 1) / SUBT;
+
+  if constexpr (KIND == SPLITTERS) {
+    for (uint32_t i = tid; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
+    __syncthreads();
+    build_spl_table<kThreads>(tbl_s, spl_s, p.logm);
+  }
+  uint8_t *mine = c8 + k1_slot(tid);
+  uint4 *c4 = reinterpret_cast<uint4 *>(c8);
+  uint32_t bad = 0;
+  auto id_of = [&](uint32_t k) -> uint32_t {
+    if constexpr (KIND == SPLITTERS) return id_spl_table(k, tbl_s, spl_s);
+    else return bucket_of_key<KIND>(k, p, spl_s);
+  };
+
+  for (uint64_t grp = blockIdx.x; grp < groups; grp += gridDim.x) {
+    const uint64_t tile = grp * SUBT + h;
+    const uint64_t base = tile * T;
+    const uint32_t nt = tile < L ? (uint32_t)umin64(T, n - base) : 0u;
+    // issue this thread's loads first (they overlap the counter reset)
+    uint4 v[KPT / 4];
+    const bool full = (nt == T);
+    if (full) {
+      const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
+#pragma unroll
+      for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * NTS + tl);  // coalesced 128-bit loads
+    }
+    if (grp == blockIdx.x) {
+      pdl_trigger();  // K2 (launched with PDL) may be scheduled once every K1 CTA has started
+      // K2's look-back status words are cleared here (K1 precedes K2 in the stream).
+      for (uint32_t i = blockIdx.x * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
+    } else {
+      __syncthreads();  // the previous group's row sums have read the counters
+    }
+    for (uint32_t i = tid; i < m * 16; i += kThreads) c4[i] = make_uint4(0, 0, 0, 0);
+    __syncthreads();
+
+    if (full) {
+      if constexpr (KIND == IDS) {
+#pragma unroll
+        for (int j = 0; j < KPT / 4; ++j) {
+          const uint64_t i0 = base + 4ull * (j * NTS + tl);
+          uint32_t raw[4];
+          if (p.id_bytes == 1) {
+            uint32_t w = __ldg(reinterpret_cast<const uint32_t *>((const uint8_t *)ids + i0));
+            raw[0] = w & 255u; raw[1] = (w >> 8) & 255u; raw[2] = (w >> 16) & 255u; raw[3] = w >> 24;
+          } else {
+            uint4 w = __ldg(reinterpret_cast<const uint4 *>((const uint32_t *)ids + i0));
+            raw[0] = w.x; raw[1] = w.y; raw[2] = w.z; raw[3] = w.w;
+          }
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            bad |= raw[q] > p.mmask;
+            mine[min(raw[q], p.mmask) * kThreads] += 1;
+          }
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < KPT / 4; ++j) {
+          mine[id_of(v[j].x) * kThreads] += 1;
+          mine[id_of(v[j].y) * kThreads] += 1;
+          mine[id_of(v[j].z) * kThreads] += 1;
+          mine[id_of(v[j].w) * kThreads] += 1;
+        }
+      }
+    } else {
+      for (uint32_t i = tl; i < nt; i += NTS) {
+        uint32_t id;
+        if constexpr (KIND == IDS) {
+          uint32_t raw = p.id_bytes == 1 ? (uint32_t)((const uint8_t *)ids)[base + i]
+                                         : ((const uint32_t *)ids)[base + i];
+          bad |= raw > p.mmask;
+          id = min(raw, p.mmask);
+        } else {
+          id = id_of(keys[base + i]);
+        }
+        mine[id * kThreads] += 1;
+      }
+    }
+    __syncthreads();
+
+    // tile column j = the bytes of row j that belong to this tile's threads;
+    // thread j (< m) of each half sums its 256/SUBT bytes with dp4a, reading
+    // 16-byte chunks in a lane-rotated order (conflict-free)
+    constexpr int CPH = 16 / SUBT;  // 16-byte chunks per half-row
+    for (uint32_t b = tl; b < m && tile < L; b += NTS) {
+      const uint4 *row = c4 + b * 16 + h * CPH;
+      uint32_t acc = 0;
+#pragma unroll
+      for (int j = 0; j < CPH; ++j) {
+        const uint4 w = row[(j + b) & (CPH - 1)];
+        acc = __dp4a(w.x, 0x01010101u, acc);
+        acc = __dp4a(w.y, 0x01010101u, acc);
+        acc = __dp4a(w.z, 0x01010101u, acc);
+        acc = __dp4a(w.w, 0x01010101u, acc);
+      }
+      H[(uint64_t)b * L + tile] = acc;
+    }
+  }
+  if constexpr (KIND == IDS) {
+    if (p.validate && __any_sync(0xFFFFFFFFu, bad) && lane == 0) atomicOr(err_flag, 1u);
+  }
+}
+
 // ============================================================== K2 scan
 // G = exclusive scan of row-vectorised H (in place), Alg. 1 P:825-828:
 // G[j][l] = sum_{k<j} sum_l' h_{k,l'} + sum_{l'<l} h_{j,l'} (terms 1+2 of

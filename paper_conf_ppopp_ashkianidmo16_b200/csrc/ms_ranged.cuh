@@ -72,7 +72,8 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   constexpr int KPT = 16, S = NT1 * KPT, FLUSH = 255 / KPT;
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t *spl_s = smem;                                              // kMaxM words (SPLITTERS)
-  uint32_t *acc = smem + (KIND == SPLITTERS ? kMaxM : 0);              // [32]
+  uint32_t *tbl_s = smem + kMaxM;                                      // kSplBins words (SPLITTERS)
+  uint32_t *acc = smem + (KIND == SPLITTERS ? kMaxM + kSplBins : 0);   // [32]
   uint8_t *c8 = reinterpret_cast<uint8_t *>(acc + 32);                // [m][NT1]
   const uint32_t tid = threadIdx.x, lane = tid & 31;
   const uint32_t m = p.m;
@@ -85,6 +86,8 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   if (tid < 32) acc[tid] = 0;
   if constexpr (KIND == SPLITTERS) {
     for (uint32_t i = tid; i < (1u << p.logm); i += NT1) spl_s[i] = p.spl[i];
+    __syncthreads();
+    build_spl_table<NT1>(tbl_s, spl_s, p.logm);
   }
   __syncthreads();
   uint8_t *mine = c8 + k1r_slot<NT1>(tid);
@@ -95,15 +98,15 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
       bad |= raw > p.mmask;
       id = min(raw, p.mmask);
     } else {
-      id = bucket_of_key<KIND>(raw, p, spl_s);
+      id = KIND == SPLITTERS ? id_spl_table(raw, tbl_s, spl_s) : bucket_of_key<KIND>(raw, p, spl_s);
     }
     mine[id * NT1] += 1;
   };
 
   int since = 0;
   uint64_t base = k0;
-  for (; base + S <= k1; base += S) {  // full sub-tiles: chunk g = j*NT1 + tid holds keys 4g..4g+3
-    if constexpr (KIND == IDS) {
+  if constexpr (KIND == IDS) {
+    for (; base + S <= k1; base += S) {  // full sub-tiles: chunk g = j*NT1 + tid holds keys 4g..4g+3
       if (p.id_bytes == 1) {  // 16 ids per thread = one 16-byte chunk
         const uint4 w = __ldg(reinterpret_cast<const uint4 *>((const uint8_t *)ids + base) + tid);
         const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
@@ -117,17 +120,23 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
 #pragma unroll
         for (int j = 0; j < KPT / 4; ++j) { count(v[j].x); count(v[j].y); count(v[j].z); count(v[j].w); }
       }
-    } else {
+      if (++since == FLUSH) {
+        k1r_flush<NT1>(c8, acc, m);
+        since = 0;
+      }
+    }
+  } else {
+    for (; base + S <= k1; base += S) {  // full sub-tiles: chunk g = j*NT1 + tid holds keys 4g..4g+3
       uint4 v[KPT / 4];
       const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * NT1 + tid);
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) { count(v[j].x); count(v[j].y); count(v[j].z); count(v[j].w); }
-    }
-    if (++since == FLUSH) {
-      k1r_flush<NT1>(c8, acc, m);
-      since = 0;
+      if (++since == FLUSH) {
+        k1r_flush<NT1>(c8, acc, m);
+        since = 0;
+      }
     }
   }
   if (base < k1) {  // last, partial sub-tile: whole 16-byte chunks where they fit, scalar keys after
@@ -166,7 +175,7 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
 }
 
 inline size_t k1r_smem(uint32_t m, int kind, int nt1) {
-  return (kind == SPLITTERS ? kMaxM * 4 : 0) + 32 * 4 + (size_t)m * nt1;
+  return (kind == SPLITTERS ? (kMaxM + kSplBins) * 4 : 0) + 32 * 4 + (size_t)m * nt1;
 }
 
 // ============================================================== K2r
