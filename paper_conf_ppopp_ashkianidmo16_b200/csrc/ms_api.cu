@@ -147,15 +147,17 @@ template <int KIND>
 cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const void *ids,
                       uint32_t n, uint32_t *H, uint64_t *zero_ptr, uint32_t zero_words,
                       uint32_t *flag, cudaStream_t s) {
-  const size_t smem = k1_smem(p->spec.m, KIND);
+  const size_t smem = p->spec.m > 32 ? (kMaxM + kWarps * (size_t)p->spec.m) * 4 : k1_smem(p->spec.m, KIND);
   // one CTA per tile group; SPLITTERS: k1s_prescan on a persistent grid (8 CTAs
   // per SM) so the bin table is built once per CTA
 #define MS_K1(KPT, SUBT)                                                                          \
   {                                                                                                \
-    auto k = KIND == SPLITTERS ? k1s_prescan<KIND, KPT, SUBT> : k1_prescan<KIND, KPT, SUBT>;      \
+    auto k = p->spec.m > 32     ? k1a_prescan<KIND, KPT, SUBT>                                     \
+             : KIND == SPLITTERS ? k1s_prescan<KIND, KPT, SUBT>                                     \
+                                 : k1_prescan<KIND, KPT, SUBT>;                                     \
     set_smem(k, smem);                                                                             \
     uint64_t grid = (g.L + SUBT - 1) / SUBT;                                                       \
-    if (KIND == SPLITTERS) grid = std::min<uint64_t>(grid, 8ull * (uint64_t)sm_count());           \
+    if (KIND == SPLITTERS && p->spec.m <= 32) grid = std::min<uint64_t>(grid, 8ull * (uint64_t)sm_count()); \
     k<<<(unsigned)grid, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, zero_words, \
                                              flag);                                                \
   }

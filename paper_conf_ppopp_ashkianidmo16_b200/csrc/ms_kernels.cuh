@@ -132,6 +132,98 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   }
 }
 
+// K1 for m > 32: per-warp u32 histograms in shared memory updated with
+// shared-memory atomics (RED.ADD), summed over the tile's warps.  The byte-
+// counter form above zeroes and reduces m * 256 bytes per tile (64 KB at
+// m = 256, 16 B per key); this one touches 8 * m words (2 B per key).
+template <int KIND, int KPT, int SUBT>
+__global__ void __launch_bounds__(kThreads)
+k1a_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
+            uint32_t L, uint32_t *__restrict__ H, const __grid_constant__ BucketParams p,
+            uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
+  constexpr int NTS = kThreads / SUBT;   // threads per tile
+  constexpr int T = NTS * KPT;           // keys per tile
+  constexpr int WPTILE = kWarps / SUBT;  // warps per tile
+  extern __shared__ __align__(16) uint32_t smem[];
+  uint32_t *spl_s = smem;                // kMaxM words (SPLITTERS)
+  uint32_t *hist = smem + kMaxM;         // [kWarps][m]
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t h = tid / NTS, tl = tid % NTS;
+  const uint64_t tile = (uint64_t)blockIdx.x * SUBT + h;
+  const uint64_t base = tile * T;
+  const uint32_t nt = tile < L ? (uint32_t)umin64(T, n - base) : 0u;
+  const uint32_t m = p.m;
+
+  uint4 v[KPT / 4];
+  const bool full = (nt == T);
+  if (full && KIND != IDS) {
+    const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
+#pragma unroll
+    for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * NTS + tl);
+  }
+  pdl_trigger();
+  for (uint32_t i = blockIdx.x * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
+  for (uint32_t i = tid; i < kWarps * m; i += kThreads) hist[i] = 0;
+  if constexpr (KIND == SPLITTERS) {
+    for (uint32_t i = tid; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
+  }
+  __syncthreads();
+  uint32_t *hw = hist + warp * m;
+  uint32_t bad = 0;
+  if (full) {
+    if constexpr (KIND == IDS) {
+#pragma unroll
+      for (int j = 0; j < KPT / 4; ++j) {
+        const uint64_t i0 = base + 4ull * (j * NTS + tl);
+        uint32_t raw[4];
+        if (p.id_bytes == 1) {
+          uint32_t w = __ldg(reinterpret_cast<const uint32_t *>((const uint8_t *)ids + i0));
+          raw[0] = w & 255u; raw[1] = (w >> 8) & 255u; raw[2] = (w >> 16) & 255u; raw[3] = w >> 24;
+        } else {
+          uint4 w = __ldg(reinterpret_cast<const uint4 *>((const uint32_t *)ids + i0));
+          raw[0] = w.x; raw[1] = w.y; raw[2] = w.z; raw[3] = w.w;
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          bad |= raw[q] > p.mmask;
+          atomicAdd(hw + min(raw[q], p.mmask), 1u);
+        }
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < KPT / 4; ++j) {
+        atomicAdd(hw + bucket_of_key<KIND>(v[j].x, p, spl_s), 1u);
+        atomicAdd(hw + bucket_of_key<KIND>(v[j].y, p, spl_s), 1u);
+        atomicAdd(hw + bucket_of_key<KIND>(v[j].z, p, spl_s), 1u);
+        atomicAdd(hw + bucket_of_key<KIND>(v[j].w, p, spl_s), 1u);
+      }
+    }
+  } else {
+    for (uint32_t i = tl; i < nt; i += NTS) {
+      uint32_t id;
+      if constexpr (KIND == IDS) {
+        uint32_t raw = p.id_bytes == 1 ? (uint32_t)((const uint8_t *)ids)[base + i]
+                                       : ((const uint32_t *)ids)[base + i];
+        bad |= raw > p.mmask;
+        id = min(raw, p.mmask);
+      } else {
+        id = bucket_of_key<KIND>(keys[base + i], p, spl_s);
+      }
+      atomicAdd(hw + id, 1u);
+    }
+  }
+  if constexpr (KIND == IDS) {
+    if (p.validate && __any_sync(0xFFFFFFFFu, bad) && lane == 0) atomicOr(err_flag, 1u);
+  }
+  __syncthreads();
+  for (uint32_t b = tl; b < m && tile < L; b += NTS) {
+    uint32_t acc = 0;
+#pragma unroll
+    for (int w = 0; w < WPTILE; ++w) acc += hist[(h * WPTILE + w) * m + b];
+    H[(uint64_t)b * L + tile] = acc;
+  }
+}
+
 // Persistent form of K1 for MS_SPLITTERS: the bin table (ms_device.cuh) is
 // built once per CTA, then the CTA walks tile groups with a stride of gridDim.x.
 template <int KIND, int KPT, int SUBT>
