@@ -58,7 +58,7 @@ keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"]
 units = {"gpu__time_duration.sum": 1.0}
 for f in sorted(os.listdir(src)):
-    m = re.match(rf"prof_{tag}_(\w+?)_(k1_prescan|k2_scan|k3p_postscan|k3_postscan)\.ncu-rep$", f)
+    m = re.match(rf"prof_{tag}_(\w+?)_(k1_prescan|k1r_prescan|k1s_prescan|k1a_prescan|k2_scan|k2r_scan|k3v_postscan|k3p_postscan|k3_postscan)\.ncu-rep$", f)
     if not m:
         continue
     cfg, kern = m.group(1), m.group(2)
@@ -69,10 +69,10 @@ for f in sorted(os.listdir(src)):
     get = lambda k: (float(d[h.index(k)]), u[h.index(k)]) if k in h else (None, "")  # noqa: E731
 
     def to_bytes(v, unit):
-        return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
+        return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}.get(unit, 1)
 
     t, tu = get("gpu__time_duration.sum")
-    t_us = t * {"nsecond": 1e-3, "usecond": 1, "msecond": 1e3}.get(tu, 1)
+    t_us = t * {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1, "us": 1, "msecond": 1e3, "ms": 1e3}.get(tu, 1)
     rd, rdu = get("dram__bytes_read.sum")
     wr, wru = get("dram__bytes_write.sum")
     dram = to_bytes(rd, rdu) + to_bytes(wr, wru)
