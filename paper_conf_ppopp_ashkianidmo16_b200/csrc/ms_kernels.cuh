@@ -461,13 +461,18 @@ __global__ void __launch_bounds__(kThreads)
 k_bucket_ids(const uint32_t *__restrict__ keys, uint64_t n, uint32_t *__restrict__ out,
              const __grid_constant__ BucketParams p) {
   __shared__ uint32_t spl_s[kMaxM];
-  if constexpr (KIND == SPLITTERS) {
+  __shared__ uint32_t tbl_s[KIND == SPLITTERS ? kSplBins : 1];
+  if constexpr (KIND == SPLITTERS) {  // the same bin table as K1 / K3 (so the functor tests pin it)
     for (uint32_t i = threadIdx.x; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
+    __syncthreads();
+    build_spl_table<kThreads>(tbl_s, spl_s, p.logm);
     __syncthreads();
   }
   for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n;
-       i += (uint64_t)gridDim.x * kThreads)
-    out[i] = bucket_of_key<KIND>(keys[i], p, spl_s);
+       i += (uint64_t)gridDim.x * kThreads) {
+    if constexpr (KIND == SPLITTERS) out[i] = id_spl_table(keys[i], tbl_s, spl_s);
+    else out[i] = bucket_of_key<KIND>(keys[i], p, spl_s);
+  }
 }
 
 }  // namespace ms

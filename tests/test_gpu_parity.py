@@ -217,6 +217,14 @@ def _clustered_splitter_sets():
         half = (m - 1) // 2
         mix = [int(x) for x in rng.integers(0, 1 << 32, half)] + [0xA0FFFFFF] * ((m - 1) - half)
         sets.append(sorted(mix))
+    # the 1024-bin table of K1/K3 (bins of 2^22 keys, ms_device.cuh id_spl_table):
+    # many splitters in one bin, splitters on bin starts, on the last and the
+    # second-to-last key of a bin, and runs of duplicates inside one bin
+    for m in (3, 32, 256):
+        sets.append(sorted(int(x) for x in rng.integers(0x12C00000, 0x12C00000 + (1 << 22), m - 1)))
+        sets.append(sorted(int(t) << 22 for t in rng.integers(0, 1024, m - 1)))
+        sets.append(sorted((int(t) << 22) + (1 << 22) - 1 - int(t % 2) for t in rng.integers(0, 1024, m - 1)))
+        sets.append(sorted([0x40000005] * ((m - 1) // 2) + [int(x) for x in rng.integers(0, 1 << 32, m - 1 - (m - 1) // 2)]))
     sets.append([0])
     sets.append([0xFFFFFFFF])
     sets.append([0, 0xFFFFFFFF, 0xFFFFFFFF])
@@ -227,7 +235,7 @@ def test_splitter_functor_clustered():
     P = _pkg()
     for spl in _clustered_splitter_sets():
         near = {s + d for s in spl for d in (-1, 0, 1) if 0 <= s + d <= 0xFFFFFFFF}
-        near |= {(t << 24) + d for t in range(256) for d in (-1, 0, 1) if 0 <= (t << 24) + d <= 0xFFFFFFFF}
+        near |= {(t << 22) + d for t in range(1024) for d in (-2, -1, 0, 1) if 0 <= (t << 22) + d <= 0xFFFFFFFF}
         kn = np.array(sorted(near | {0xFFFFFFFF}), dtype=np.uint32)
         plan = P.Plan(P.BucketSpec.from_splitters(spl), len(kn))
         got = from_dev(plan.bucket_ids(to_dev(kn)))

@@ -14,7 +14,7 @@ import bench  # noqa: E402
 from paper_conf_ppopp_ashkianidmo16_b200 import model  # noqa: E402
 
 tag = sys.argv[1]
-src = os.path.join(ROOT, "gpurun_out")
+src = os.environ.get("PROF_SRC", os.path.join(ROOT, "gpurun_out"))
 out = []
 
 
@@ -37,7 +37,7 @@ if os.path.exists(lp):
         a = agg.setdefault(k, [0, 0.0])
         a[0] += 1
         a[1] += v
-    ours = {k: v for k, v in agg.items() if k.startswith(("k1_", "k2_", "k3", "k_"))}
+    ours = {k: v for k, v in agg.items() if re.match(r"k[0-9_]", k)}
     tot = sum(v[1] for v in ours.values())
     out.append(f"## Launch list (`ncu --metrics gpu__time_duration.sum --clock-control none`, "
                f"`python bench.py --steps 3 --warmup 3 --no-extra --no-cpu`, config {bench.DEFAULT})\n")
@@ -49,7 +49,8 @@ if os.path.exists(lp):
     out.append("")
 
 # (2) full captures
-traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+PROF_OUT = os.environ.get("PROF_OUT", os.path.join(ROOT, "profiles"))
+traffic_path = os.path.join(PROF_OUT, "ncu_traffic.json")
 traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
 keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__issue_active.avg.pct_of_peak_sustained_active",
@@ -96,8 +97,8 @@ for f in sorted(os.listdir(src)):
         traffic[cfg] = int(dram)
 with open(traffic_path, "w") as fh:
     json.dump(traffic, fh, indent=1, sort_keys=True)
-os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
-with open(os.path.join(ROOT, "profiles", f"{tag}_summary.md"), "w") as fh:
+os.makedirs(PROF_OUT, exist_ok=True)
+with open(os.path.join(PROF_OUT, f"{tag}_summary.md"), "w") as fh:
     fh.write(f"# ncu summary, round tag {tag}\n\nGenerated by tools/summarize_profiles.py from "
              f"tools/profile_round.sh output (1 B200, clocks not locked).\n\n" + "\n".join(out) + "\n")
 print("\n".join(out))
