@@ -31,6 +31,7 @@ struct ms_plan_s {
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt (MS_K3_NT)
   int ranged = 0;  // CTA-range variant (ms_ranged.cuh, m <= 32): 0 never, 1 when L is large, 2 always
   int pdl = 1;     // programmatic dependent launch of K2, K3 (MS_PDL=0 disables)
+  int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
@@ -187,12 +188,13 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                         uint32_t *vo, uint32_t n, cudaStream_t s, int ranged = 0,
-                        uint32_t *grid_out = nullptr, int pdl = 0) {
+                        uint32_t *grid_out = nullptr, int pdl = 0, const RangeScan *rs = nullptr) {
   K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
             p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, sm_count(), s};
   a.ranged = ranged;
   a.grid_out = grid_out;
   a.pdl = pdl;
+  if (rs) a.rs = *rs;
   if (p->spec.m <= 32 && p->k3v && p->kkind != IDS) {  // K3 v2 (ms_k3_v2.cuh)
     switch (p->kkind) {
       case LOWBITS: return k3v_launch_lowbits(a);
@@ -376,6 +378,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (flags & MS_VARIANT_RANGED) p->ranged = 2;
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
+  if (const char *e = getenv("MS_RANGED_K2")) p->fuse_k2r = atoi(e) ? 0 : 1;
   *plan = p;
   return MS_OK;
 }
@@ -530,6 +533,16 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
     if (dispatch_k1r(p, g, C, keys_in, ids, (uint32_t)n, HC, flag, s) != cudaSuccess) return MS_ERR_CUDA;
     if (ev && p->tracing == 1) cudaEventRecord(ev[1], s);
     const uint32_t ksub = k1r_split(C), R = C * ksub;
+    if (p->fuse_k2r) {  // K1r -> K3 (the range scan runs in K3's prologue): two launches
+      if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
+      const RangeScan rs{HC, offsets, R, ksub};
+      if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 1, nullptr, pdl,
+                      &rs) != cudaSuccess)
+        return MS_ERR_CUDA;
+      if (ev) cudaEventRecord(ev[3], s);
+      p->last_launches = 2;
+      return MS_OK;
+    }
     const size_t smem2 = (size_t)R * p->spec.m * 4;
     set_smem(k2r_scan, smem2);
     if (launch_ex(pdl, k2r_scan, dim3(1), dim3(kR2Threads), smem2, s, (const uint32_t *)HC, GB, R, ksub, p->spec.m,

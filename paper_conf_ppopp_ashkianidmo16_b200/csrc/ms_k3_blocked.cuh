@@ -404,7 +404,7 @@ __global__ void __launch_bounds__(NT, NT == 256 ? (KV ? 2 : 3) : (KV ? 4 : 6))
 k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const void *__restrict__ ids, const uint32_t *__restrict__ G,
              uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
-             uint32_t L, const __grid_constant__ BucketParams p) {
+             uint32_t L, const __grid_constant__ BucketParams p, const __grid_constant__ RangeScan rs) {
   using Ly = K3pLayout<LOGMP, KV, IDS8, KPT, NT>;
   constexpr int T = Ly::T, STAGES = Ly::STAGES, CW = Ly::CW, MP = Ly::MP, K = Ly::K;
   constexpr int LOGNT = NT == 256 ? 8 : 7;
@@ -452,7 +452,12 @@ k3p_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ val
   uint32_t grun = 0;   // RANGED: G_row of the current tile (all threads of bucket row `row`)
   if constexpr (RANGED) {
     const uint32_t row = tid >> (LOGNT - LOGMP);
-    if (iters && row < m) grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
+    if (rs.HC != nullptr) {  // K2r folded in (the reorder slots are free until tile 0)
+      grun = range_base<NT, LOGMP>(rs, m, blockIdx.x, n, sm + Ly::O_KEYS, row);
+      __syncthreads();
+    } else if (iters && row < m) {
+      grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
+    }
   } else {
     if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
   }
@@ -528,7 +533,7 @@ inline cudaError_t k3p_launch_one(Kern k, size_t smem, const K3pArgs &a) {
     return cudaSuccess;
   }
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, a.keys, a.vals, a.ids, a.G,
-                                  a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+                                  a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

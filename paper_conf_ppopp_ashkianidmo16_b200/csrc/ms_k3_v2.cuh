@@ -82,7 +82,8 @@ __global__ void __launch_bounds__(NT, MINB)
 k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv,
              const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const uint32_t *__restrict__ G, uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
-             uint32_t n, uint32_t L, const __grid_constant__ BucketParams p) {
+             uint32_t n, uint32_t L, const __grid_constant__ BucketParams p,
+             const __grid_constant__ RangeScan rs) {
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES>;
   constexpr int MP = Ly::MP, K = Ly::K, T = Ly::T, TB = Ly::TB, RS = Ly::RS;
   constexpr int NW = NT / 32;
@@ -163,7 +164,12 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   uint32_t grun = 0;   // RANGED: G_row of the current tile (all threads of bucket row `row`)
   const uint32_t row = tid >> (LOGNT - LOGMP);
   if constexpr (RANGED) {
-    if (iters && row < m) grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
+    if (rs.HC != nullptr) {  // K2r folded in: this range's G from K1r's rows (keys_s is free until tile 0)
+      grun = range_base<NT, LOGMP>(rs, m, blockIdx.x, n, keys_s, row);
+      __syncthreads();
+    } else if (iters && row < m) {
+      grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
+    }
   } else {
     if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
   }
@@ -463,7 +469,7 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   if (!make_tile_map(&tmk, a.keys, rows, Ly::T) || !make_tile_map(&tmv, KV ? a.vals : nullptr, rows, Ly::T))
     return cudaErrorInvalidValue;
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals,
-                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp);
+                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

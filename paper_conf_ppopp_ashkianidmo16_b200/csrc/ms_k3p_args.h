@@ -11,6 +11,15 @@
 
 namespace ms {
 
+// Ranged variant with the range scan folded into K3 (range_base below):
+// HC = K1r's R = C*k sub-range rows of m counts; offsets written by CTA 0.
+// HC == nullptr: K3 reads GB[c][:] written by K2r instead.
+struct RangeScan {
+  const uint32_t *HC;
+  uint32_t *offsets;
+  uint32_t R, k;
+};
+
 struct K3pArgs {
   const uint32_t *keys, *vals;
   const void *ids;
@@ -24,6 +33,7 @@ struct K3pArgs {
   int ranged = 0;               // 1: CTA-range mode (G = GB[C][m], ms_ranged.cuh); m <= 32 only
   int pdl = 0;                  // 1: programmatic dependent launch after K2 (ms_device.cuh pdl_wait)
   uint32_t *grid_out = nullptr;  // non-null: only compute the grid C (no launch)
+  RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged: fold K2r into K3's prologue when rs.HC is set
 };
 
 // Launch with cudaLaunchAttributeProgrammaticStreamSerialization when `pdl`:
@@ -44,6 +54,59 @@ inline cudaError_t launch_ex(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 b
   cfg.numAttrs = pdl ? 1 : 0;
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
+
+// ============================================================== K2r folded into K3
+// Terms 1+2 of Eq. (2) for range c, computed redundantly by every K3 CTA from
+// K1r's rows (replaces the K2r launch and its hand-off; the R x m words are
+// L2-resident, R*m*4 <= 76 KB for m <= 16):
+//   pre_j = sum_{r < c*k} HC[r][j],  tot_j = sum_r HC[r][j],
+//   GB[c][j] = sum_{i<j} tot_i + pre_j,  offsets[j] = sum_{i<j} tot_i (CTA 0).
+// Thread (s, j) (j = tid mod MP) sums rows s, s + NS, ... of column j, so one
+// warp load covers 32/MP consecutive rows (contiguous words when m = MP).
+// Every thread of the CTA must call it; `red` is 2*NT words of scratch shared
+// memory that nothing else touches until the caller's next __syncthreads().
+// Returns GB[c][row] (0 for row >= m).
+template <int NT, int LOGMP>
+__device__ __forceinline__ uint32_t range_base(const RangeScan &rs, uint32_t m, uint32_t c, uint32_t n,
+                                               uint32_t *red, uint32_t row) {
+  constexpr uint32_t MP = 1u << LOGMP, NS = NT / MP;
+  const uint32_t tid = threadIdx.x, j = tid & (MP - 1), s = tid >> LOGMP;
+  const uint32_t cut = c * rs.k;
+  uint32_t pre = 0, post = 0;
+  if (j < m) {
+    const uint32_t *col = rs.HC + j;
+#pragma unroll 8
+    for (uint32_t r = s; r < rs.R; r += NS) {
+      const uint32_t v = __ldcg(col + (uint64_t)r * m);
+      if (r < cut) pre += v;
+      else post += v;
+    }
+  }
+  red[tid] = pre;
+  red[NT + tid] = post;
+  __syncthreads();
+#pragma unroll
+  for (uint32_t d = NS / 2; d >= 1; d >>= 1) {
+    if (s < d) {
+      red[tid] += red[tid + d * MP];
+      red[NT + tid] += red[NT + tid + d * MP];
+    }
+    __syncthreads();
+  }
+  if (tid < 32) {
+    const uint32_t pj = tid < m ? red[tid] : 0u;
+    const uint32_t tot = tid < m ? pj + red[NT + tid] : 0u;
+    const uint32_t start = warp_incl_scan(tot, tid) - tot;
+    if (tid < m) red[NT + tid] = start + pj;
+    if (c == 0 && rs.offsets != nullptr) {
+      if (tid < m) rs.offsets[tid] = start;
+      if (tid == 0) rs.offsets[m] = n;
+    }
+  }
+  __syncthreads();
+  return row < m ? red[NT + row] : 0u;
+}
+
 
 constexpr uint32_t kMaxRanges = 1024;  // upper bound on the CTA-range count C (workspace sizing)
 

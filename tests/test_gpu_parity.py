@@ -66,11 +66,15 @@ def test_parity_matrix(kind, m, variant):
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} n={n} kv={kv} {variant}")
 
 
+@pytest.mark.parametrize("k2r", [False, True])
 @pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("ids", 5, True),
-                                       ("lowbits", 2, False), ("delta", 32, True)])
-def test_ranged_range_edges(kind, m, kv):
+                                       ("lowbits", 2, False), ("delta", 32, True), ("delta", 16, True)])
+def test_ranged_range_edges(kind, m, kv, k2r, monkeypatch):
     """Ranged variant around C = resident K3 CTAs: L < C, L = C +- 1, L = 3C + r (ranges of 1..4 tiles,
-    the ragged last tile at the end of the last range)."""
+    the ragged last tile at the end of the last range); the range scan folded into K3's prologue
+    (default) and as a separate K2r launch (MS_RANGED_K2=1)."""
+    if k2r:
+        monkeypatch.setenv("MS_RANGED_K2", "1")
     P = _pkg()
     probe = P.Plan(P.BucketSpec(**make_case(kind, m, 1, 0, kv=kv)["spec_kw"]), 1 << 24, with_values=kv,
                    variant="ranged")
