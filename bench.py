@@ -320,7 +320,63 @@ def measure_e2e(cfg, plan, keys_d, vals_d, K):
     return n / (ms * 1e-3) / 1e9, h2d, d2h, ms
 
 
-def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True):
+def torch_bucket_ids(cfg, keys):
+    """Bucket ids with plain torch ops (the comparator's own pre-pass; not our kernels)."""
+    import torch
+    k = keys.to(torch.int64) & 0xFFFFFFFF
+    if cfg["kind"] == "lowbits":
+        return (k >> cfg.get("shift", 0)) & (cfg["m"] - 1)
+    if cfg["kind"] == "delta":
+        return torch.clamp(k // cfg["delta"], max=cfg["m"] - 1)
+    spl = torch.as_tensor(W.gen_splitters(cfg["m"], cfg["seed"]).astype(np.int64), device=keys.device)
+    return torch.searchsorted(spl, k, side="left")  # #{j : s_j < k}
+
+
+def measure_comparators(cfg, plan, keys, vals, K, flush):
+    """Same-run comparators, each timed with CUDA events on the current stream, L2 flushed
+    before every run: (i) torch.sort of the keys (+ gather of the values): the paper's radix-sort row
+    (Table 3/6); (ii) the reduced-bit sort: ids by torch elementwise ops, torch.sort(ids,
+    stable=True), gather keys (and values) -- its output must be bit-identical to ours."""
+    import torch
+    s = torch.cuda.current_stream()
+    ko = torch.empty_like(keys)
+    vo = torch.empty_like(vals) if vals is not None else None
+    plan.run(keys, vals, keys_out=ko, vals_out=vo)
+
+    def sort_keys():
+        sk, idx = torch.sort(keys)
+        if vals is not None:
+            return sk, vals[idx]
+        return sk, None
+
+    def reduced_bit():
+        ids = torch_bucket_ids(cfg, keys).to(torch.uint8 if cfg["m"] <= 256 else torch.int32)
+        _, idx = torch.sort(ids, stable=True)
+        return keys[idx], (vals[idx] if vals is not None else None)
+
+    out = {}
+    for nm, fn in (("torch_sort_keys", sort_keys), ("torch_sort_on_bucket_id", reduced_bit)):
+        res = fn()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(K):
+            flush()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            fn()
+            e1.record(s)
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        ms = statistics.median(ts)
+        out[nm] = {"value": round(keys.numel() / (ms * 1e-3) / 1e9, 3), "unit": "G keys/s", "ms": round(ms, 4)}
+        if nm == "torch_sort_on_bucket_id":
+            same = bool(torch.equal(res[0], ko)) and (vals is None or bool(torch.equal(res[1], vo)))
+            out[nm]["bit_identical_to_multisplit"] = same
+        del res
+    return out
+
+
+def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparators=False):
     import torch
     import paper_conf_ppopp_ashkianidmo16_b200 as P
     from paper_conf_ppopp_ashkianidmo16_b200 import model
@@ -359,6 +415,11 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True):
         "gpu_launches": launches * K, "tile": T, "tiles": L, "variant": variant,
         "clocks": clocks.result(),
     }
+    if comparators:
+        comp = measure_comparators(cfg, plan, keys, vals, max(3, min(K, 10)), flush)
+        for v in comp.values():
+            v["multisplit_speedup"] = round(value / v["value"], 2)
+        res["comparators"] = comp
     if with_e2e:
         e2e_v, h2d, d2h, e2e_ms = measure_e2e(cfg, plan, keys, vals, max(2, min(K, 5)))
         res["e2e"] = {"value": e2e_v * world, "unit": "G keys/s", "h2d_bytes_per_step": h2d,
@@ -455,7 +516,8 @@ def run_ours(args, cfg, world, rank, local):
         b.build()
     barrier(world)
     # the per-rank kernels, traced (roofline, stages); at N = 1 this IS the headline step
-    res = bench_config(args.config, cfg, args.steps, args.warmup, device, world, rank, with_e2e=(world == 1))
+    res = bench_config(args.config, cfg, args.steps, args.warmup, device, world, rank, with_e2e=(world == 1),
+                       comparators=(world == 1 and not args.no_extra))
     if world > 1:
         d = bench_dist(args.config, cfg, args.steps, args.warmup, device, world, rank, args.dist_backend)
         local_value = res["value"]
@@ -466,12 +528,14 @@ def run_ours(args, cfg, world, rank, local):
     if not args.no_extra and world == 1:
         for nm in args.extra.split(","):
             if nm and nm in CONFIGS and nm != args.config:
-                r = bench_config(nm, CONFIGS[nm], max(5, args.steps // 4), 3, device, world, rank, with_e2e=False)
+                r = bench_config(nm, CONFIGS[nm], max(5, args.steps // 4), 3, device, world, rank, with_e2e=False,
+                                 comparators=True)
                 extra[nm] = {"desc": CONFIGS[nm]["desc"], "value": round(r["value"], 2),
                              "ms_per_step": round(r["ms_per_step"], 4),
                              "whole_step_frac": round(r["whole_step_frac"], 4),
                              "k3_frac": r["roofline"]["frac"], "k1_frac": r["roofline"]["k1_prescan_frac"],
-                             "stages_ms": {k: round(v, 4) for k, v in r["stages_ms"].items()}}
+                             "stages_ms": {k: round(v, 4) for k, v in r["stages_ms"].items()},
+                             "comparators": r.get("comparators")}
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = time_oracle(cfg, budget_s=10.0)
@@ -498,6 +562,8 @@ def run_ours(args, cfg, world, rank, local):
             "whole_step_hbm_gbs": round(res["whole_step_hbm_gbs"], 1),
             "tile": res["tile"], "variant": res["variant"], "extra": extra,
         }
+        if "comparators" in res:
+            out["comparators"] = res["comparators"]
         if "local_step" in res:
             out["local_step"] = res["local_step"]
         print(json.dumps(out), flush=True)
