@@ -15,7 +15,7 @@ CSRC = os.path.join(HERE, "csrc")
 OBJ = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libms.so")
 SOURCES = ["ms_api.cu", "ms_dist.cu", "k3p_lowbits.cu", "k3p_shiftc.cu", "k3p_shift.cu", "k3p_delta.cu", "k3p_splitters.cu", "k3p_ids.cu"]
-HEADERS = ["ms_k3_v2.cuh", "ms_kernels.cuh", "ms_device.cuh", "ms_k3_blocked.cuh", "ms_k3_warp.cuh", "ms_k3p_args.h", "ms_ranged.cuh"]
+HEADERS = ["ms_k3_v2.cuh", "ms_kernels.cuh", "ms_device.cuh", "ms_k3_blocked.cuh", "ms_k3_warp.cuh", "ms_k3p_args.h", "ms_ranged.cuh", "ms_k3_lsd.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr"]

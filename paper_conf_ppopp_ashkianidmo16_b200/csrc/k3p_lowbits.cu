@@ -3,9 +3,11 @@
 #include "ms_k3_blocked.cuh"
 #include "ms_k3_warp.cuh"
 #include "ms_k3_v2.cuh"
+#include "ms_k3_lsd.cuh"
 
 namespace ms {
 cudaError_t k3p_launch_lowbits(const K3pArgs &a) { return k3p_launch<LOWBITS>(a); }
 cudaError_t k3w_launch_lowbits(const K3pArgs &a) { return k3w_launch<LOWBITS>(a); }
 cudaError_t k3v_launch_lowbits(const K3pArgs &a) { return k3v_launch<LOWBITS>(a); }
+cudaError_t k3h_launch_lowbits(const K3pArgs &a) { return k3h_launch<LOWBITS>(a); }
 }  // namespace ms

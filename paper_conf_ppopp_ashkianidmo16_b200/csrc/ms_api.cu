@@ -31,6 +31,9 @@ struct ms_plan_s {
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt (MS_K3_NT)
   int ranged = 0;  // CTA-range variant (ms_ranged.cuh, m <= 32): 0 never, 1 when L is large, 2 always
   int pdl = 1;     // programmatic dependent launch of K2, K3 (MS_PDL=0 disables)
+  // 32 < m <= 256, kinds other than MS_IDS: MS_K3H=1 selects the two-digit K3
+  // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
+  int k3h = 0;
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
   int32_t last_launches;
@@ -75,8 +78,9 @@ uint64_t delta_magic(uint32_t d) { return ~0ull / d + 1; }
 // Rounds per warp R (tile T = 256 R): 16 for m <= 32, 32 above (runs of T/m
 // keys stay >= 32 keys = 128 B); halved while the grid would not fill two
 // waves of 148 SMs (small n is launch/latency bound, not HBM bound).
-int rounds_for(uint32_t m, uint64_t n, uint32_t kpt) {
+int rounds_for(uint32_t m, uint64_t n, uint32_t kpt, bool k3h) {
   if (m <= 32) return (int)kpt;  // blocked-rank K3: T = 256 * kpt for every n
+  if (k3h) return 16;            // persistent two-digit K3 (ms_k3_lsd.cuh): T = 4096 for every n
   int R = 16;
   while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
   return R;
@@ -94,7 +98,7 @@ struct Geometry {
 
 Geometry geometry(const ms_plan_s *p, uint64_t n) {
   Geometry g{};
-  g.R = rounds_for(p->spec.m, n, p->kpt * p->k3nt / 256);
+  g.R = rounds_for(p->spec.m, n, p->kpt * p->k3nt / 256, p->k3h && p->kkind != IDS);
   g.T = 256u * g.R;
   g.L = (n + g.T - 1) / g.T;
   g.hg_words = (uint64_t)p->spec.m * g.L;
@@ -212,6 +216,15 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
       case DELTA: return k3p_launch_delta(a);
       case SPLITTERS: return k3p_launch_splitters(a);
       default: return k3p_launch_ids(a);
+    }
+  }
+  if (p->k3h && p->kkind != IDS) {  // 32 < m <= 256: two-digit local multisplit (ms_k3_lsd.cuh)
+    switch (p->kkind) {
+      case LOWBITS: return k3h_launch_lowbits(a);
+      case SHIFTC: return k3h_launch_shiftc(a);
+      case SHIFT: return k3h_launch_shift(a);
+      case DELTA: return k3h_launch_delta(a);
+      default: return k3h_launch_splitters(a);
     }
   }
   switch (p->kkind) {  // m > 32: warp-ballot K3 (ms_k3_warp.cuh)
@@ -378,6 +391,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (flags & MS_VARIANT_RANGED) p->ranged = 2;
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
+  if (const char *e = getenv("MS_K3H")) p->k3h = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_RANGED_K2")) p->fuse_k2r = atoi(e) ? 0 : 1;
   *plan = p;
   return MS_OK;

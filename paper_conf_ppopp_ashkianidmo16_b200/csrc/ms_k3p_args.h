@@ -122,6 +122,12 @@ cudaError_t k3v_launch_shiftc(const K3pArgs &a);
 cudaError_t k3v_launch_shift(const K3pArgs &a);
 cudaError_t k3v_launch_delta(const K3pArgs &a);
 cudaError_t k3v_launch_splitters(const K3pArgs &a);
+// 32 < m <= 256, kinds other than MS_IDS: two-digit LSD local multisplit (ms_k3_lsd.cuh)
+cudaError_t k3h_launch_lowbits(const K3pArgs &a);
+cudaError_t k3h_launch_shiftc(const K3pArgs &a);
+cudaError_t k3h_launch_shift(const K3pArgs &a);
+cudaError_t k3h_launch_delta(const K3pArgs &a);
+cudaError_t k3h_launch_splitters(const K3pArgs &a);
 // m > 32: warp-ballot K3 (ms_k3_warp.cuh); kpt carries the rounds per warp R (8 or 16)
 cudaError_t k3w_launch_lowbits(const K3pArgs &a);
 cudaError_t k3w_launch_shiftc(const K3pArgs &a);

@@ -87,6 +87,21 @@ def test_ranged_range_edges(kind, m, kv, k2r, monkeypatch):
             _assert_equal(case, _run_case(case, "ranged"), _expect(case), f"{kind} m={m} L={L} n={n}")
 
 
+@pytest.mark.parametrize("kind", ["lowbits", "delta", "splitters"])
+@pytest.mark.parametrize("m", [33, 64, 127, 256])
+def test_parity_two_digit_k3(kind, m, monkeypatch):
+    """The two-digit (LSD 16 x 16) K3 for m > 32, an ablation kept behind MS_K3H=1: bit-exact on ragged
+    sizes, skewed buckets and a multi-wave n."""
+    if kind == "lowbits" and m & (m - 1):
+        pytest.skip("low-bit buckets need a power-of-two m (reading #10)")
+    monkeypatch.setenv("MS_K3H", "1")
+    for i, (n, dist) in enumerate([(1, "uniform"), (4095, "uniform"), (4097, "hot"), (100003, "binomial"),
+                                   ((1 << 22) + 5, "uniform")]):
+        for kv in (False, True):
+            case = make_case(kind, m, n, seed=300 + 10 * m + i, dist=dist, kv=kv)
+            _assert_equal(case, _run_case(case), _expect(case), f"k3h {kind} m={m} n={n} {dist} kv={kv}")
+
+
 @pytest.mark.parametrize("kv", [False, True])
 def test_parity_2p28_m32(kv):
     """Headline size n = 2^28, m = 32 (DELTA 2^27, the NS configs), full element-wise compare."""
