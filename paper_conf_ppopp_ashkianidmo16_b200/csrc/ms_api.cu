@@ -374,6 +374,8 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
   if (const char *e = getenv("MS_K3_REVERSE")) p->bp.reverse = atoi(e) ? 1u : 0u;
   if (const char *e = getenv("MS_K3_NT")) p->k3nt = atoi(e) == 128 ? 128u : 256u;
+  // K3 v2 at 128 threads runs 32 keys per thread (same T = 4096)
+  if (kkind != IDS && p->k3nt == 128) p->kpt = 32;
   // variant: CTA ranges for m <= 32 when a tile's mean bucket
   // run is >= 256 keys (1 KB).  With shorter runs the strided tile walk wins:
   // its concurrently processed tiles write ADJACENT runs of every bucket (m

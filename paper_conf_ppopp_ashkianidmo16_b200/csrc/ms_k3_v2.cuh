@@ -36,10 +36,10 @@
 
 namespace ms {
 
-template <int LOGMP, bool KV, int NT, int STAGES>
+template <int LOGMP, bool KV, int NT, int STAGES, int KPT = 16>
 struct K3vLayout {
   static constexpr int MP = 1 << LOGMP;         // bucket rows (m rounded up to a power of 2, >= 2)
-  static constexpr int K = 16;                  // keys per thread (one contiguous block)
+  static constexpr int K = KPT;                 // keys per thread (one contiguous block): 16, or 32 with NT = 128
   static constexpr int T = NT * K;              // keys per tile
   static constexpr int TB = T * 4;              // bytes of one staged array (keys or values)
   static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // reorder slots incl. alignment padding
@@ -77,16 +77,17 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *tm, in
       : "memory");
 }
 
-template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB>
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB, int KPT>
 __global__ void __launch_bounds__(NT, MINB)
 k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv,
              const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const uint32_t *__restrict__ G, uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
              uint32_t n, uint32_t L, const __grid_constant__ BucketParams p,
              const __grid_constant__ RangeScan rs) {
-  using Ly = K3vLayout<LOGMP, KV, NT, STAGES>;
+  using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
   constexpr int MP = Ly::MP, K = Ly::K, T = Ly::T, TB = Ly::TB, RS = Ly::RS;
   constexpr int NW = NT / 32;
+  constexpr int NCH = K / 4;  // 16-byte chunks per thread block
   constexpr int LOGNT = NT == 256 ? 8 : 7;
   constexpr bool KEEP_ID = KIND == SPLITTERS;  // the table lookup is kept, not repeated
   extern __shared__ uint8_t smraw[];
@@ -107,10 +108,11 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   // counter words of a row (32 banks) whatever their ids; the staged block is
   // row beta >> 1, half beta & 1 of the swizzled 128-byte rows
   const uint32_t beta = 2 * lane + (warp & 1) + 64 * (warp >> 1);
-  const uint32_t srow = beta >> 1, shalf = beta & 1;
-  uint32_t choff[4];  // byte offsets of the block's 4 chunks inside a stage (128B swizzle)
+  // (K = 32: the block is the whole swizzled row beta)
+  const uint32_t srow = K == 16 ? beta >> 1 : beta, shalf = K == 16 ? beta & 1 : 0;
+  uint32_t choff[NCH];  // byte offsets of the block's chunks inside a stage (128B swizzle)
 #pragma unroll
-  for (int c = 0; c < 4; ++c) choff[c] = srow * 128 + 16 * ((4 * shalf + c) ^ (srow & 7));
+  for (int c = 0; c < NCH; ++c) choff[c] = srow * 128 + 16 * ((NCH * shalf + c) ^ (srow & 7));
   const uint32_t m = p.m;
   const uint32_t b0 = beta * K;
   // c[j][beta] at shared address ccol + j * RS
@@ -206,23 +208,23 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 
     // ---- 1. this thread's block -> registers; sequential counting into the
     // private counter column (the value read is the key's rank in the block)
-    uint4 kx[4];
+    uint4 kx[NCH];
     if constexpr (FULL) {
       mbar_wait(bar_k + st, ph);
       const uint8_t *sk = sm + Ly::O_SK + st * TB;
 #pragma unroll
-      for (int c = 0; c < 4; ++c) kx[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
+      for (int c = 0; c < NCH; ++c) kx[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
     } else {
       uint32_t t[K];
 #pragma unroll
       for (int q = 0; q < K; ++q) t[q] = b0 + q < nt ? __ldg(keys + base + b0 + q) : 0u;
 #pragma unroll
-      for (int c = 0; c < 4; ++c) kx[c] = make_uint4(t[4 * c], t[4 * c + 1], t[4 * c + 2], t[4 * c + 3]);
+      for (int c = 0; c < NCH; ++c) kx[c] = make_uint4(t[4 * c], t[4 * c + 1], t[4 * c + 2], t[4 * c + 3]);
     }
-    uint32_t rk[4];                     // ranks (< 16), one byte each
-    uint32_t idk[KEEP_ID ? 4 : 1];      // kept ids, one byte each
+    uint32_t rk[NCH];                   // ranks (< K), one byte each
+    uint32_t idk[KEEP_ID ? NCH : 1];    // kept ids, one byte each
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
+    for (int c = 0; c < NCH; ++c) {
       const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
       rk[c] = 0u;
       if constexpr (KEEP_ID) idk[c] = 0u;
@@ -329,23 +331,23 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     __syncthreads();
 
     // ---- 3. local multisplit of the tile into shared memory
-    uint4 vy[KV ? 4 : 1];
+    uint4 vy[KV ? NCH : 1];
     if constexpr (KV) {
       if constexpr (FULL) {
         mbar_wait(bar_v + st, ph);
         const uint8_t *sv = sm + Ly::O_SV + st * TB;
 #pragma unroll
-        for (int c = 0; c < 4; ++c) vy[c] = *reinterpret_cast<const uint4 *>(sv + choff[c]);
+        for (int c = 0; c < NCH; ++c) vy[c] = *reinterpret_cast<const uint4 *>(sv + choff[c]);
       } else {
         uint32_t t[K];
 #pragma unroll
         for (int q = 0; q < K; ++q) t[q] = b0 + q < nt ? __ldg(vals + base + b0 + q) : 0u;
 #pragma unroll
-        for (int c = 0; c < 4; ++c) vy[c] = make_uint4(t[4 * c], t[4 * c + 1], t[4 * c + 2], t[4 * c + 3]);
+        for (int c = 0; c < NCH; ++c) vy[c] = make_uint4(t[4 * c], t[4 * c + 1], t[4 * c + 2], t[4 * c + 3]);
       }
     }
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
+    for (int c = 0; c < NCH; ++c) {
       const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
       uint32_t vv[4];
       if constexpr (KV) {
@@ -449,9 +451,11 @@ inline bool make_tile_map(CUtensorMap *tm, const uint32_t *ptr, uint64_t rows, u
 
 template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED>
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
-  using Ly = K3vLayout<LOGMP, KV, NT, STAGES>;
-  constexpr int MINB = NT == 256 ? (KV ? 2 : 3) : (KV ? 4 : 6);
-  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB>;
+  // NT = 128 runs 32 keys per thread (same 4096-key tile, half the counter matrix per key)
+  constexpr int KPT = NT == 128 ? 32 : 16;
+  using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
+  constexpr int MINB = NT == 256 ? (KV ? 2 : 3) : (KV ? 3 : 4);
+  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
