@@ -126,32 +126,16 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
       }
     }
   } else {
-    // full sub-tiles: chunk g = j*NT1 + tid holds keys 4g..4g+3; the next
-    // sub-tile's four loads are issued before this one is counted (128 B in
-    // flight per thread: short K1r grids are latency-bound, not HBM-bound)
-    uint4 v[KPT / 4];
-    if (base + S <= k1) {
+    for (; base + S <= k1; base += S) {  // full sub-tiles: chunk g = j*NT1 + tid holds keys 4g..4g+3
+      uint4 v[KPT / 4];
       const uint4 *k4 = reinterpret_cast<const uint4 *>(keys + base);
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) v[j] = __ldg(k4 + j * NT1 + tid);
-    }
-    for (; base + S <= k1; base += S) {
-      uint4 nx[KPT / 4];
-      const bool more = base + 2 * S <= k1;
-      if (more) {
-        const uint4 *n4 = reinterpret_cast<const uint4 *>(keys + base + S);
-#pragma unroll
-        for (int j = 0; j < KPT / 4; ++j) nx[j] = __ldg(n4 + j * NT1 + tid);
-      }
 #pragma unroll
       for (int j = 0; j < KPT / 4; ++j) { count(v[j].x); count(v[j].y); count(v[j].z); count(v[j].w); }
       if (++since == FLUSH) {
         k1r_flush<NT1>(c8, acc, m);
         since = 0;
-      }
-      if (more) {
-#pragma unroll
-        for (int j = 0; j < KPT / 4; ++j) v[j] = nx[j];
       }
     }
   }

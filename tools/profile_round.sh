@@ -11,7 +11,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
   --log-file gpurun_out/prof_${TAG}_launches.csv python bench.py --steps 3 --warmup 3 --no-extra --no-cpu \
   > gpurun_out/prof_${TAG}_launches_bench.log 2>&1
 # (2) one full capture per hot kernel (K1, K2, K3) on the headline config
-for k in k1r_prescan k2r_scan k3v_postscan; do
+for k in k1r_prescan k3v_postscan; do
   timeout 300 ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 \
     -o gpurun_out/prof_${TAG}_${CFG}_$k python tools/run_case.py $CFG 2 > /dev/null 2>&1
 done
