@@ -206,6 +206,50 @@ ms_status ms_dist_pieces(int32_t nranks, int32_t rank, uint32_t m, const uint64_
                          int32_t recv_cap, int32_t *n_recv, uint64_t *offsets_global,
                          uint64_t *win_start, uint64_t *win_len);
 
+/* ---------------------------------------------------------------------------
+ * Fused sharded scatter: instead of a local output plus an
+ * exchange, the post-scan kernel stores every bucket run straight into the
+ * windows of the ranks that own it -- over NVLink / NVSwitch when the window
+ * pointers are peer mappings (CUDA IPC / symmetric memory), so the transfer
+ * overlaps the local reorder tile by tile and the local output is never
+ * written.  Same windows and the same global result as ms_dist_pieces.
+ *
+ * ms_dist_targets (HOST function): from the all-gathered counts (P*m u64, row
+ * g = rank g) compute for rank `rank`:
+ *   delta[b]     = global position - local position of its local bucket b
+ *                  (B[b] + sum_{g'<g} h[g'][b] - off_g[b]), b < m (u64[m]);
+ *   win_start[r] = first global position of rank r's window, r <= P
+ *                  (win_start[P] = N; u64[P+1]).
+ * MS_ERR_INVALID_ARG on bad sizes.
+ *
+ * ms_postscan_scatter: the post-scan (K3) of the 3-kernel path with the
+ * stores redirected: keys_in / vals_in (NULL = key-only) are this rank's shard
+ * (n local keys), G the output of ms_scan on it (m*L u32, workspace as for
+ * ms_run); every key goes to keys_dst[r][x - win_start[r]] (and the value to
+ * vals_dst[r][...]) where x = local position + delta[bucket] and r owns x.
+ * The window pointers must be dereferenceable from the calling GPU (its own
+ * memory or peer-mapped memory) and 16-byte aligned; the call is
+ * stream-ordered and the stores are complete when the kernel completes on
+ * `stream` (the CALLER synchronises the ranks before reading the windows).
+ * Supported for plans with m <= 32 and a computed bucket kind (not MS_IDS);
+ * else MS_ERR_UNSUPPORTED. nranks in 1..MS_MAX_PEERS.
+ * ------------------------------------------------------------------------- */
+#define MS_MAX_PEERS 8
+typedef struct {
+  int32_t nranks;
+  int32_t pad_;
+  uint32_t *keys_dst[MS_MAX_PEERS];
+  uint32_t *vals_dst[MS_MAX_PEERS];
+  uint64_t win_start[MS_MAX_PEERS + 1];
+  uint64_t delta[32];
+} ms_scatter_target;
+
+ms_status ms_dist_targets(int32_t nranks, int32_t rank, uint32_t m, const uint64_t *counts, uint64_t *delta,
+                          uint64_t *win_start);
+ms_status ms_postscan_scatter(ms_plan_t plan, const uint32_t *keys_in, const uint32_t *vals_in,
+                              const uint32_t *G, uint64_t n, const ms_scatter_target *target, void *workspace,
+                              size_t workspace_bytes, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -30,7 +30,21 @@ EXPORTS = [
     "ms_plan_workspace_size_host", "ms_run_host", "ms_prescan", "ms_scan", "ms_postscan",
     "ms_bucket_ids", "ms_plan_check", "ms_plan_destroy", "ms_status_string",
     "ms_plan_last_launches", "ms_plan_trace", "ms_plan_trace_read", "ms_dist_pieces",
+    "ms_dist_targets", "ms_postscan_scatter",
 ]
+
+MS_MAX_PEERS = 8
+
+
+class ms_scatter_target(ctypes.Structure):
+    _fields_ = [
+        ("nranks", ctypes.c_int32),
+        ("pad_", ctypes.c_int32),
+        ("keys_dst", ctypes.c_void_p * MS_MAX_PEERS),
+        ("vals_dst", ctypes.c_void_p * MS_MAX_PEERS),
+        ("win_start", ctypes.c_uint64 * (MS_MAX_PEERS + 1)),
+        ("delta", ctypes.c_uint64 * 32),
+    ]
 
 
 class ms_bucket_spec(ctypes.Structure):
@@ -81,6 +95,8 @@ def lib():
     L.ms_plan_trace_read.argtypes = [P, P, I32, ctypes.POINTER(I32), ctypes.POINTER(I32)]
     L.ms_dist_pieces.argtypes = [I32, I32, U32, P, P, I32, ctypes.POINTER(I32), P, I32, ctypes.POINTER(I32), P,
                                  ctypes.POINTER(U64), ctypes.POINTER(U64)]
+    L.ms_dist_targets.argtypes = [I32, I32, U32, P, P, P]
+    L.ms_postscan_scatter.argtypes = [P, P, P, P, U64, ctypes.POINTER(ms_scatter_target), P, SZ, P]
     for name in EXPORTS:
         f = getattr(L, name)
         if name != "ms_status_string":

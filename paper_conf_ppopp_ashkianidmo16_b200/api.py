@@ -217,6 +217,14 @@ class Plan:
                                      _ptr(vals_out), n, _ptr(ws), ws.numel(), _stream(stream)), "ms_postscan")
         return keys_out, vals_out
 
+    def postscan_scatter(self, keys, G, target, vals=None, workspace=None, stream=None):
+        """ms_postscan_scatter: K3 storing every run into its owners' windows (`target`: an
+        _abi.ms_scatter_target with window pointers valid on this GPU)."""
+        n = keys.numel()
+        ws = self.workspace(n) if workspace is None else workspace
+        check(_abi.lib().ms_postscan_scatter(self._h, _ptr(keys), _ptr(vals), _ptr(G), n, ctypes.byref(target),
+                                             _ptr(ws), ws.numel(), _stream(stream)), "ms_postscan_scatter")
+
     def bucket_ids(self, keys, out=None, stream=None):
         import torch
         if out is None:

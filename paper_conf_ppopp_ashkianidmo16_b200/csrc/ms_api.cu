@@ -454,7 +454,7 @@ ms_status ms_prescan(ms_plan_t p, const uint32_t *keys_in, const void *ids, uint
                      uint32_t *H, void *ws, size_t ws_bytes, void *stream) {
   ms_status st = check_common(p, keys_in, ids, n);
   if (st != MS_OK) return st;
-  if (!H) return MS_ERR_INVALID_ARG;
+  if (!H && n > 0) return MS_ERR_INVALID_ARG;
   if (misaligned(H)) return MS_ERR_ALIGNMENT;
   Geometry g;
   if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
@@ -501,6 +501,47 @@ ms_status ms_postscan(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals
   if (n == 0) return MS_OK;
   cudaError_t e = dispatch_k3(p, g, keys_in, vals_in, ids, G, keys_out, vals_out, (uint32_t)n,
                               (cudaStream_t)stream);
+  return e == cudaSuccess ? MS_OK : MS_ERR_CUDA;
+}
+
+ms_status ms_postscan_scatter(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, const uint32_t *G,
+                              uint64_t n, const ms_scatter_target *t, void *ws, size_t ws_bytes, void *stream) {
+  if (!p) return MS_ERR_INVALID_ARG;
+  if (p->spec.m > 32 || p->kkind == IDS || !p->k3v) return MS_ERR_UNSUPPORTED;
+  ms_status st = check_common(p, keys_in, nullptr, n);
+  if (st != MS_OK) return st;
+  if (!t || t->nranks < 1 || t->nranks > MS_MAX_PEERS) return MS_ERR_INVALID_ARG;
+  if (vals_in && !p->kv) return MS_ERR_UNSUPPORTED;
+  if (misaligned(vals_in) || misaligned(G)) return MS_ERR_ALIGNMENT;
+  for (int32_t r = 0; r < t->nranks; ++r) {
+    if (t->win_start[r + 1] < t->win_start[r]) return MS_ERR_INVALID_ARG;
+    const bool empty = t->win_start[r + 1] == t->win_start[r];
+    if (!empty && (!t->keys_dst[r] || (vals_in && !t->vals_dst[r]))) return MS_ERR_INVALID_ARG;
+    if (misaligned(t->keys_dst[r]) || misaligned(t->vals_dst[r])) return MS_ERR_ALIGNMENT;
+  }
+  Geometry g;
+  if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
+  if (n == 0) return MS_OK;
+  if (!G) return MS_ERR_INVALID_ARG;
+  DistTarget d{};
+  d.P = t->nranks;
+  for (int32_t r = 0; r < t->nranks; ++r) {
+    d.keys[r] = t->keys_dst[r];
+    d.vals[r] = t->vals_dst[r];
+  }
+  for (int32_t r = 0; r <= t->nranks; ++r) d.wst[r] = t->win_start[r];
+  for (uint32_t b = 0; b < p->spec.m; ++b) d.delta[b] = t->delta[b];
+  K3pArgs a{keys_in, vals_in, nullptr, G, nullptr, nullptr, (uint32_t)n, (uint32_t)g.L, p->spec.m,
+            p->spec.id_bytes, p->kpt, p->k3nt, &p->bp, sm_count(), (cudaStream_t)stream};
+  a.ds = &d;
+  cudaError_t e;
+  switch (p->kkind) {
+    case LOWBITS: e = k3v_launch_lowbits(a); break;
+    case SHIFTC: e = k3v_launch_shiftc(a); break;
+    case SHIFT: e = k3v_launch_shift(a); break;
+    case DELTA: e = k3v_launch_delta(a); break;
+    default: e = k3v_launch_splitters(a); break;
+  }
   return e == cudaSuccess ? MS_OK : MS_ERR_CUDA;
 }
 

@@ -86,3 +86,24 @@ extern "C" ms_status ms_dist_pieces(int32_t P, int32_t rank, uint32_t m, const u
   *n_recv = nr;
   return MS_OK;
 }
+
+extern "C" ms_status ms_dist_targets(int32_t P, int32_t rank, uint32_t m, const uint64_t *counts, uint64_t *delta,
+                                     uint64_t *win_start) {
+  if (P < 1 || P > MS_MAX_PEERS || rank < 0 || rank >= P || m < 1 || !counts || !delta || !win_start)
+    return MS_ERR_INVALID_ARG;
+  // B[b] + sum_{g'<rank} h[g'][b] - off_rank[b], off_rank = exclusive scan of h[rank]
+  uint64_t B = 0, off = 0;
+  for (uint32_t b = 0; b < m; ++b) {
+    uint64_t col = 0, pref = 0;
+    for (int32_t g = 0; g < P; ++g) {
+      if (g == rank) pref = col;
+      col += counts[(size_t)g * m + b];
+    }
+    delta[b] = B + pref - off;  // >= 0: B >= off (all ranks' lower buckets include mine)
+    B += col;
+    off += counts[(size_t)rank * m + b];
+  }
+  const Windows W{B / (uint64_t)P, B % (uint64_t)P};
+  for (int32_t r = 0; r <= P; ++r) win_start[r] = W.start(r);
+  return MS_OK;
+}

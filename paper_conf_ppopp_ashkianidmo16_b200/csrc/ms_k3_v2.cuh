@@ -83,7 +83,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
              const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
              const uint32_t *__restrict__ G, uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
              uint32_t n, uint32_t L, const __grid_constant__ BucketParams p,
-             const __grid_constant__ RangeScan rs) {
+             const __grid_constant__ RangeScan rs, const __grid_constant__ DistTarget ds) {
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
   constexpr int MP = Ly::MP, K = Ly::K, T = Ly::T, TB = Ly::TB, RS = Ly::RS;
   constexpr int NW = NT / 32;
@@ -307,7 +307,17 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       grun += rtot;
       if ((tid & (TPR - 1)) == 0) Gj[row] = Gr;
     } else {
-      Gr = row < m ? Gj[row] : 0u;
+      Gr = row < m ? Gj[row] : 0u;  // (fused sharded scatter: replaced by the destination offset below)
+    }
+    if constexpr (!RANGED) {
+      // fused sharded scatter: align the run to its destination offset in the
+      // window that owns its first key (global position G_j + delta_j)
+      if (ds.P > 0 && row < m) {
+        const uint64_t gs = (uint64_t)Gr + ds.delta[row];
+        uint32_t r = 0;
+        for (int i = 1; i < ds.P; ++i) r += gs >= ds.wst[i] ? 1u : 0u;
+        Gr = (uint32_t)(gs - ds.wst[r]);
+      }
     }
     // padded run start P_j = S_j + 3j + ((G_j - S_j - 3j) & 3): P_j = G_j (mod 4)
     // and P_j >= P_{j-1} + h_{j-1}; closed form, no serial dependency over j
@@ -378,7 +388,50 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 
     // ---- 4. bucket runs: SPB threads per bucket share its <= 3 head keys,
     // <= 3 tail keys and the TMA bulk store(s) of the 16-byte-aligned body
-    {
+    if (!RANGED && ds.P > 0) {
+      // fused sharded scatter: the run [gs, gs + len) of global positions is
+      // cut at window boundaries; each piece goes to its owner's window, the
+      // 16-byte-aligned body by one TMA bulk store per array (peer memory is
+      // plain global memory to the TMA), the rest by the SPB threads
+      constexpr uint32_t SPB = NT / 32;
+      const uint32_t b = tid / SPB, sub = tid % SPB;
+      if (b < m) {
+        uint32_t left = rowS[b + 1] - rowS[b];
+        uint32_t src = Pj[b];
+        uint64_t gs = (uint64_t)Gj[b] + ds.delta[b];
+        while (left) {
+          uint32_t r = 0;
+          for (int i = 1; i < ds.P; ++i) r += gs >= ds.wst[i] ? 1u : 0u;
+          const uint64_t room = ds.wst[r + 1] - gs;
+          const uint32_t len = room < left ? (uint32_t)room : left;
+          const uint64_t doff = gs - ds.wst[r];
+          uint32_t *dk = ds.keys[r] + doff;
+          uint32_t *dv = KV ? ds.vals[r] + doff : nullptr;
+          uint32_t head = min(len, (4u - (uint32_t)(doff & 3u)) & 3u);
+          uint32_t body = (len - head) & ~3u;
+          if (((src + head) & 3u) != 0u) {  // source and destination disagree mod 16 B: no bulk copy
+            head = len;
+            body = 0;
+          }
+          for (uint32_t i = sub; i < head; i += SPB) {
+            dk[i] = keys_s[src + i];
+            if constexpr (KV) dv[i] = vals_s[src + i];
+          }
+          for (uint32_t i = head + body + sub; i < len; i += SPB) {
+            dk[i] = keys_s[src + i];
+            if constexpr (KV) dv[i] = vals_s[src + i];
+          }
+          if (body && (sub == SPB - 1 || (KV && sub == SPB - 2))) {
+            if (sub == SPB - 1) bulk_s2g(dk + head, keys_s + src + head, body * 4u);
+            else bulk_s2g(dv + head, vals_s + src + head, body * 4u);
+            bulk_commit();
+          }
+          gs += len;
+          src += len;
+          left -= len;
+        }
+      }
+    } else {
       constexpr uint32_t SPB = NT / 32;
       const uint32_t b = tid / SPB, sub = tid % SPB;
       if (b < m) {
@@ -418,7 +471,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   const uint32_t iters_full = iters - (has_tail ? 1u : 0u);
   for (uint32_t it = 0; it < iters_full; ++it) tile_body(it, std::true_type{});
   if (has_tail) tile_body(iters_full, std::false_type{});
-  bulk_wait_read0();
+  if (ds.P > 0) bulk_wait0();  // peer stores complete before the grid ends (made visible by the stream order)
+  else bulk_wait_read0();
 }
 
 // ------------------------------------------------------------------ host launcher
@@ -473,7 +527,8 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   if (!make_tile_map(&tmk, a.keys, rows, Ly::T) || !make_tile_map(&tmv, KV ? a.vals : nullptr, rows, Ly::T))
     return cudaErrorInvalidValue;
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals,
-                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs);
+                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs,
+                                  a.ds ? *a.ds : DistTarget{});
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

@@ -20,6 +20,21 @@ struct RangeScan {
   uint32_t R, k;
 };
 
+// Fused sharded scatter: K3 stores every bucket
+// run straight into its owners' output windows -- peer memory over NVLink on a
+// multi-GPU box (pointers from CUDA IPC / symmetric memory), or any device
+// pointers.  Rank r owns global positions [wst[r], wst[r+1]); the local run of
+// bucket j at local position x goes to global position x + delta[j].  P = 0:
+// plain local output (keys_out / vals_out).
+constexpr int kMaxPeers = 8;
+struct DistTarget {
+  uint32_t *keys[kMaxPeers];
+  uint32_t *vals[kMaxPeers];
+  uint64_t wst[kMaxPeers + 1];
+  uint64_t delta[32];  // m <= 32 (K3 v2)
+  int32_t P;
+};
+
 struct K3pArgs {
   const uint32_t *keys, *vals;
   const void *ids;
@@ -34,6 +49,7 @@ struct K3pArgs {
   int pdl = 0;                  // 1: programmatic dependent launch after K2 (ms_device.cuh pdl_wait)
   uint32_t *grid_out = nullptr;  // non-null: only compute the grid C (no launch)
   RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged: fold K2r into K3's prologue when rs.HC is set
+  const DistTarget *ds = nullptr;           // fused sharded scatter (K3 v2, tile variant only)
 };
 
 // Launch with cudaLaunchAttributeProgrammaticStreamSerialization when `pdl`:

@@ -103,3 +103,123 @@ def dist_multisplit(keys, vals=None, spec=None, group=None, local=None):
         for req in dist.batch_isend_irecv(ops):
             req.wait()
     return out_k, out_v, offg, ws
+
+
+# ---------------------------------------------------------------------------
+# Fused sharded scatter (include/ms.h ms_postscan_scatter):
+# K1 + K2 locally, the count all-gather, then ONE post-scan kernel that stores
+# every bucket run straight into the owners' windows (peer memory over
+# NVLink/NVSwitch) -- no local output, no staging copy, no send/recv.
+def dist_targets(nranks: int, rank: int, m: int, counts):
+    """Host planning (ms_dist_targets): counts (P x m) -> (delta u64[m], win_start u64[P+1])."""
+    counts = np.ascontiguousarray(counts, dtype=np.uint64)
+    assert counts.shape == (nranks, m)
+    delta = np.zeros(m, dtype=np.uint64)
+    wst = np.zeros(nranks + 1, dtype=np.uint64)
+    check(_abi.lib().ms_dist_targets(nranks, rank, m, counts.ctypes.data_as(ctypes.c_void_p),
+                                     delta.ctypes.data_as(ctypes.c_void_p), wst.ctypes.data_as(ctypes.c_void_p)),
+          "ms_dist_targets")
+    return delta, wst
+
+
+def scatter_target(keys_ptrs, vals_ptrs, win_start, delta):
+    """ms_scatter_target from per-rank window base pointers (device addresses valid on this GPU)."""
+    P = len(keys_ptrs)
+    if not 1 <= P <= _abi.MS_MAX_PEERS:
+        raise ValueError(f"fused scatter supports 1..{_abi.MS_MAX_PEERS} ranks, got {P}")
+    t = _abi.ms_scatter_target()
+    t.nranks = P
+    for r in range(P):
+        t.keys_dst[r] = int(keys_ptrs[r]) or None
+        t.vals_dst[r] = (int(vals_ptrs[r]) or None) if vals_ptrs is not None else None
+    for r in range(P + 1):
+        t.win_start[r] = int(win_start[r])
+    for b, d in enumerate(delta):
+        t.delta[b] = int(d)
+    return t
+
+
+def _local_scan(plan, keys, ws):
+    """K1 + K2 on this rank's shard: (G = m*L u32 matrix, counts u64[m] on the host)."""
+    import torch
+    n = keys.numel()
+    off = torch.empty(plan.spec.m + 1, dtype=torch.int32, device=keys.device)
+    G = plan.prescan(keys, workspace=ws)
+    plan.scan(G, n, offsets=off, workspace=ws)
+    o = off.cpu().numpy().view(np.uint32).astype(np.uint64)
+    return G, o[1:] - o[:-1]
+
+
+def _fused_plan(spec, n, with_values):
+    from .api import Plan
+    if spec.m > 32 or spec.kind == "ids":
+        raise NotImplementedError("the fused sharded scatter runs on K3 v2 (m <= 32, computed bucket ids)")
+    return Plan(spec, max(n, 1), with_values=with_values, variant="3k")
+
+
+def scatter_multisplit_virtual(shards_keys, shards_vals=None, spec=None):
+    """P VIRTUAL ranks on one GPU, same kernels and arithmetic as dist_multisplit_fused: each
+    shard's K1+K2, then each shard's scatter-K3 writing into all P windows (here plain local
+    allocations standing in for peer mappings).  Returns (keys, vals) = the windows concatenated,
+    which equal the single-GPU stable multisplit of the concatenated shards."""
+    import torch
+    P = len(shards_keys)
+    m = spec.m
+    kv = shards_vals is not None
+    plans, scans = [], []
+    for r in range(P):
+        plan = _fused_plan(spec, shards_keys[r].numel(), kv)
+        ws = plan.workspace(shards_keys[r].numel())
+        G, cnt = _local_scan(plan, shards_keys[r], ws)
+        plans.append((plan, ws))
+        scans.append((G, cnt))
+    counts = np.stack([c for _, c in scans])
+    dev = shards_keys[0].device
+    _, wst = dist_targets(P, 0, m, counts)
+    wins_k = [torch.empty(max(int(wst[r + 1] - wst[r]), 4), dtype=torch.int32, device=dev) for r in range(P)]
+    wins_v = [torch.empty_like(w) for w in wins_k] if kv else None
+    for r in range(P):
+        delta, _ = dist_targets(P, r, m, counts)
+        t = scatter_target([w.data_ptr() for w in wins_k], [w.data_ptr() for w in wins_v] if kv else None, wst, delta)
+        plan, ws = plans[r]
+        plan.postscan_scatter(shards_keys[r], scans[r][0], t, vals=shards_vals[r] if kv else None, workspace=ws)
+    torch.cuda.synchronize()
+    keys = torch.cat([wins_k[r][:int(wst[r + 1] - wst[r])] for r in range(P)])
+    vals = torch.cat([wins_v[r][:int(wst[r + 1] - wst[r])] for r in range(P)]) if kv else None
+    return keys, vals
+
+
+def dist_multisplit_fused(keys, vals=None, spec=None, group=None):
+    """Collective, one process per GPU (NCCL process group): like dist_multisplit, but the
+    exchange IS the post-scan kernel: windows are symmetric-memory buffers mapped on every peer
+    (torch.distributed._symmetric_memory over NVLink/NVSwitch) and each rank's K3 stores its
+    runs straight into them.  Returns (keys_window, vals_window, win_start)."""
+    import torch
+    import torch.distributed as dist
+    import torch.distributed._symmetric_memory as symm_mem
+    P = dist.get_world_size(group)
+    g = dist.get_rank(group)
+    m = spec.m
+    kv = vals is not None
+    plan = _fused_plan(spec, keys.numel(), kv)
+    ws = plan.workspace(keys.numel())
+    G, cnt = _local_scan(plan, keys, ws)
+    c = torch.as_tensor(cnt.astype(np.int64), device=keys.device)
+    gathered = torch.empty(P * m, dtype=torch.int64, device=keys.device)
+    dist.all_gather_into_tensor(gathered, c, group=group)
+    counts = gathered.cpu().numpy().astype(np.uint64).reshape(P, m)
+    delta, wst = dist_targets(P, g, m, counts)
+    wmax = max(int(wst[r + 1] - wst[r]) for r in range(P)) or 4
+    grp = group if group is not None else dist.group.WORLD
+    bufs, ptrs = [], []
+    for _ in range(2 if kv else 1):
+        b = symm_mem.empty(wmax, dtype=torch.int32, device=keys.device)
+        h = symm_mem.rendezvous(b, grp)
+        bufs.append(b)
+        ptrs.append(list(h.buffer_ptrs))
+    t = scatter_target(ptrs[0], ptrs[1] if kv else None, wst, delta)
+    plan.postscan_scatter(keys, G, t, vals=vals, workspace=ws)
+    torch.cuda.current_stream().synchronize()
+    dist.barrier(group)  # every rank's stores into my window are complete
+    wl = int(wst[g + 1] - wst[g])
+    return bufs[0][:wl], (bufs[1][:wl] if kv else None), int(wst[g])

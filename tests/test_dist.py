@@ -17,7 +17,7 @@ import torch.multiprocessing as mp
 
 import oracle
 import workloads as W
-from paper_conf_ppopp_ashkianidmo16_b200.dist import dist_multisplit, dist_pieces
+from paper_conf_ppopp_ashkianidmo16_b200.dist import dist_multisplit, dist_pieces, dist_targets
 from paper_conf_ppopp_ashkianidmo16_b200.api import BucketSpec
 
 
@@ -53,6 +53,36 @@ def test_pieces_cover_and_match(P, m):
         assert np.all(cover == 1)
         for r in range(P):                                           # receives tile the window exactly
             assert sum(p[1] for p in plans[r][1]) == wins[r][1]
+
+
+@pytest.mark.parametrize("P,m", [(1, 1), (2, 3), (3, 32), (4, 8), (8, 32), (5, 2)])
+def test_targets_match_pieces(P, m):
+    """ms_dist_targets (fused scatter planning) agrees with ms_dist_pieces: same windows, and every
+    piece rank g sends sits at global position local position + delta[bucket of that position]."""
+    rng = np.random.default_rng(7 * P + m)
+    for trial in range(20):
+        counts = rng.integers(0, 40, size=(P, m)).astype(np.uint64)
+        if trial % 3 == 0:
+            counts[:, 0] *= 25
+        if trial % 4 == 0:
+            counts[rng.integers(P)] = 0
+        for g in range(P):
+            delta, wst = dist_targets(P, g, m, counts)
+            send, _, _, ws, wl = dist_pieces(P, g, m, counts)
+            assert wst[g] == ws and wst[g + 1] - wst[g] == wl
+            assert wst[0] == 0 and wst[P] == counts.sum()
+            off = np.concatenate([[0], np.cumsum(counts[g])]).astype(np.uint64)
+            for s_off, ln, peer, d_off in send:
+                b = int(np.searchsorted(off, s_off, side="right") - 1)
+                while counts[g][b] == 0:
+                    b += 1
+                assert int(wst[peer]) + d_off == s_off + int(delta[b])
+
+
+def test_targets_reject_bad_sizes():
+    from paper_conf_ppopp_ashkianidmo16_b200._abi import MultisplitError
+    with pytest.raises(MultisplitError):
+        dist_targets(9, 0, 4, np.zeros((9, 4), np.uint64))   # more than MS_MAX_PEERS ranks
 
 
 def test_pieces_follow_eq2():

@@ -318,3 +318,66 @@ def test_repeated_runs_same_workspace():
     for _ in range(3):
         ko, vo, off = plan.run(kd, vd)
         assert np.array_equal(from_dev(ko), exp[0]) and np.array_equal(from_dev(vo), exp[1])
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+@pytest.mark.parametrize("kind,m", [("lowbits", 2), ("delta", 8), ("splitters", 32), ("delta", 5), ("lowbits", 1)])
+def test_fused_scatter_virtual_ranks(P, kind, m):
+    """Fused sharded scatter (ms_postscan_scatter) with P virtual ranks on one GPU:
+    each shard's K3 writes its runs straight into all P windows; the windows concatenated must equal
+    the oracle's stable multisplit of the concatenated shards.  Ragged shards (empty, < 1 tile,
+    several tiles + tail), skewed buckets so window boundaries cut runs, KO and KV."""
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import scatter_multisplit_virtual
+    rng = np.random.default_rng(1000 * P + m)
+    for trial, dist in enumerate(["uniform", "hot", "binomial"]):
+        sizes = [int(x) for x in rng.integers(0, 3 * 4096 + 77, size=P)]
+        if trial == 1 and P > 1:
+            sizes[0] = 0
+        if trial == 2:
+            sizes[-1] = 4097
+        for kv in (False, True):
+            case = make_case(kind, m, sum(sizes), seed=50 + trial + 10 * P, dist=dist if m > 1 else "uniform", kv=kv)
+            P_ = _pkg()
+            spec = P_.BucketSpec(**case["spec_kw"])
+            cuts = np.concatenate([[0], np.cumsum(sizes)])
+            ks = [to_dev(case["keys"][cuts[r]:cuts[r + 1]]) for r in range(P)]
+            vs = [to_dev(case["vals"][cuts[r]:cuts[r + 1]]) for r in range(P)] if kv else None
+            ko, vo = scatter_multisplit_virtual(ks, vs, spec)
+            eko, evo, _ = _expect(case)
+            what = f"P={P} {kind} m={m} {dist} sizes={sizes} kv={kv}"
+            assert np.array_equal(from_dev(ko), eko), what
+            if kv:
+                assert np.array_equal(from_dev(vo), evo), what
+
+
+@pytest.mark.parametrize("kv", [False, True])
+def test_fused_scatter_virtual_large(kv):
+    """C5-shaped (splitters m = 32, uniform) at 2^26 keys over 4 virtual ranks, full compare."""
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import scatter_multisplit_virtual
+    n, P = 1 << 26, 4
+    case = make_case("splitters", 32, n, seed=W.SEEDS["C3"], kv=kv, vals_kind="random")
+    spec = _pkg().BucketSpec(**case["spec_kw"])
+    q = n // P
+    ks = [to_dev(case["keys"][r * q:(r + 1) * q]) for r in range(P)]
+    vs = [to_dev(case["vals"][r * q:(r + 1) * q]) for r in range(P)] if kv else None
+    ko, vo = scatter_multisplit_virtual(ks, vs, spec)
+    eko, evo, _ = _expect(case)
+    assert np.array_equal(from_dev(ko), eko)
+    if kv:
+        assert np.array_equal(from_dev(vo), evo)
+
+
+def test_fused_scatter_rejects_unsupported():
+    """m > 32 or precomputed ids: the fused scatter is K3 v2 only (MS_ERR_UNSUPPORTED)."""
+    from paper_conf_ppopp_ashkianidmo16_b200 import _abi
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import scatter_target
+    P_ = _pkg()
+    keys = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    out = torch.empty_like(keys)
+    for spec in (P_.BucketSpec.delta_range(64, 1 << 26), P_.BucketSpec.precomputed(8, 1)):
+        plan = P_.Plan(spec, 4096, variant="3k")
+        t = scatter_target([out.data_ptr()], None, [0, 4096], [0] * 32)
+        G = torch.zeros(spec.m, dtype=torch.int32, device="cuda")
+        with pytest.raises(_abi.MultisplitError) as e:
+            plan.postscan_scatter(keys, G, t)
+        assert e.value.status == _abi.MS_ERR_UNSUPPORTED
