@@ -429,7 +429,7 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparato
     return res
 
 
-def bench_dist(name, cfg, K, Wm, device, world, rank, backend):
+def bench_dist(name, cfg, K, Wm, device, world, rank, backend, mode="nccl"):
     """N > 1: the sharded multisplit (dist.py): local ms_run + count all-gather + grouped
     point-to-point exchange into balanced output windows.  Weak scaling: every rank holds
     cfg['n'] keys (global indices rank*n ...).  Time = CUDA events around each whole
@@ -437,7 +437,7 @@ def bench_dist(name, cfg, K, Wm, device, world, rank, backend):
     import torch
     import torch.distributed as dist
     import paper_conf_ppopp_ashkianidmo16_b200 as P
-    from paper_conf_ppopp_ashkianidmo16_b200.dist import dist_multisplit
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import dist_multisplit, dist_multisplit_fused
     n = cfg["n"]
     keys, vals = inputs_torch(cfg, n, rank * n, device)
     spec = spec_of(cfg)
@@ -450,9 +450,16 @@ def bench_dist(name, cfg, K, Wm, device, world, rank, backend):
             return ko.cpu(), (vo.cpu() if vo is not None else None), off.cpu()
         return ko, vo, off
 
+    if mode == "fused":  # K3 stores straight into the owners' symmetric-memory windows (NVLink peer stores)
+        def step(k, v):
+            wk, wv, w0 = dist_multisplit_fused(k, v, spec)
+            return wk, wv, None, w0
+    else:
+        def step(k, v):
+            return dist_multisplit(k, v, spec, local=local)
     flush = L2Flush(device)
     for _ in range(Wm):
-        dist_multisplit(keys, vals, spec, local=local)
+        step(keys, vals)
     torch.cuda.synchronize()
     dist.barrier()
     s = torch.cuda.current_stream()
@@ -465,7 +472,7 @@ def bench_dist(name, cfg, K, Wm, device, world, rank, backend):
             dist.barrier()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
-            wk, wv, offg, ws = dist_multisplit(keys, vals, spec, local=local)
+            wk, wv, offg, ws = step(keys, vals)
             e1.record(s)
             torch.cuda.synchronize()
             tot_ms += e0.elapsed_time(e1)
@@ -485,7 +492,7 @@ def bench_dist(name, cfg, K, Wm, device, world, rank, backend):
         e0.record(s)
         kd = kh.to(device, non_blocking=True)
         vd = vh.to(device, non_blocking=True) if vh is not None else None
-        wk, wv, offg, ws = dist_multisplit(kd, vd, spec, local=local)
+        wk, wv, offg, ws = step(kd, vd)
         wk_h = wk.to("cpu", non_blocking=True)
         wv_h = wv.to("cpu", non_blocking=True) if wv is not None else None
         e1.record(s)
@@ -519,7 +526,8 @@ def run_ours(args, cfg, world, rank, local):
     res = bench_config(args.config, cfg, args.steps, args.warmup, device, world, rank, with_e2e=(world == 1),
                        comparators=(world == 1 and not args.no_extra))
     if world > 1:
-        d = bench_dist(args.config, cfg, args.steps, args.warmup, device, world, rank, args.dist_backend)
+        d = bench_dist(args.config, cfg, args.steps, args.warmup, device, world, rank, args.dist_backend,
+                       args.dist_mode)
         local_value = res["value"]
         res.update(value=d["value"], ms_per_step=d["ms_per_step"], clocks=d["clocks"], e2e=d["e2e"])
         res["local_step"] = {"value_if_independent": round(local_value, 3),
@@ -554,7 +562,10 @@ def run_ours(args, cfg, world, rank, local):
                        "kind": cfg["kind"], "kv": cfg["kv"], "dist": cfg["dist"],
                        "l2": "flushed between timed steps (512 MiB write + 512 MiB read so the write-back is done), outside the timed kernels",
                        "parallelism": (f"sharded multisplit x{world}: local ms_run + NCCL count all-gather + "
-                                       f"grouped send/recv into balanced windows ({args.dist_backend})")
+                                       f"grouped send/recv into balanced windows ({args.dist_backend})"
+                                       if args.dist_mode == "nccl" else
+                                       f"sharded multisplit x{world}: local K1+K2 + NCCL count all-gather + fused "
+                                       f"K3 peer stores into symmetric-memory windows")
                        if world > 1 else "single GPU"},
             "roofline": res["roofline"], "e2e": res["e2e"], "cpu_baseline": cpu,
             "gpu_launches": res["gpu_launches"], "clocks": res["clocks"],
@@ -584,6 +595,9 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N>1 exchange backend (gloo: host-staged, for testing on one GPU)")
+    ap.add_argument("--dist-mode", default="nccl", choices=["nccl", "fused"],
+                    help="N>1 exchange: NCCL grouped send/recv after a local ms_run, or the fused K3 that "
+                         "stores into the owners' symmetric-memory windows (m <= 32, computed bucket ids)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -189,6 +189,9 @@ def scatter_multisplit_virtual(shards_keys, shards_vals=None, spec=None):
     return keys, vals
 
 
+_SYMM = {}
+
+
 def dist_multisplit_fused(keys, vals=None, spec=None, group=None):
     """Collective, one process per GPU (NCCL process group): like dist_multisplit, but the
     exchange IS the post-scan kernel: windows are symmetric-memory buffers mapped on every peer
@@ -211,12 +214,20 @@ def dist_multisplit_fused(keys, vals=None, spec=None, group=None):
     delta, wst = dist_targets(P, g, m, counts)
     wmax = max(int(wst[r + 1] - wst[r]) for r in range(P)) or 4
     grp = group if group is not None else dist.group.WORLD
-    bufs, ptrs = [], []
-    for _ in range(2 if kv else 1):
-        b = symm_mem.empty(wmax, dtype=torch.int32, device=keys.device)
-        h = symm_mem.rendezvous(b, grp)
-        bufs.append(b)
-        ptrs.append(list(h.buffer_ptrs))
+    # symmetric windows are allocated + rendezvoused once per (group, device, arrays) and reused
+    # while they are large enough (every rank takes the same decision: wmax is global)
+    key = (id(grp), str(keys.device), kv)
+    ent = _SYMM.get(key)
+    if ent is None or ent[0] < wmax:
+        cap = max(wmax, 4)
+        bufs, ptrs = [], []
+        for _ in range(2 if kv else 1):
+            b = symm_mem.empty(cap, dtype=torch.int32, device=keys.device)
+            h = symm_mem.rendezvous(b, grp)
+            bufs.append(b)
+            ptrs.append(list(h.buffer_ptrs))
+        ent = _SYMM[key] = (cap, bufs, ptrs)
+    _, bufs, ptrs = ent
     t = scatter_target(ptrs[0], ptrs[1] if kv else None, wst, delta)
     plan.postscan_scatter(keys, G, t, vals=vals, workspace=ws)
     torch.cuda.current_stream().synchronize()
