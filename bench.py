@@ -68,6 +68,9 @@ for _m in (2, 4, 8, 16, 32, 64, 128, 256):
             desc=f"{'key-value' if _kv else 'key-only'} m={_m} delta D=2^32/m, n=2^28, uniform", kind="delta",
             m=_m, delta=(1 << 32) // _m, n=1 << 28, kv=_kv, dist="uniform", seed=W.SEEDS["C4"])
 
+for _e in (22, 23, 24, 26, 27, 28):  # size sweep of the headline workload (fixed-cost analysis)
+    CONFIGS[f"C2_n{_e}"] = dict(CONFIGS["C2"], n=1 << _e, desc=CONFIGS["C2"]["desc"].replace("2^25", f"2^{_e}"))
+
 DEFAULT = "C2"
 
 

@@ -34,6 +34,7 @@ struct ms_plan_s {
   // 32 < m <= 256, kinds other than MS_IDS: MS_K3H=1 selects the two-digit K3
   // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
   int k3h = 0;
+  int one = 0;       // ranged variant as ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk)
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
   int32_t last_launches;
@@ -393,6 +394,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (flags & MS_VARIANT_RANGED) p->ranged = 2;
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
+  if (const char *e = getenv("MS_ONE")) p->one = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3H")) p->k3h = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_RANGED_K2")) p->fuse_k2r = atoi(e) ? 0 : 1;
   *plan = p;
@@ -581,6 +583,20 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   // K2 and K3 use programmatic dependent launch unless per-stage events sit
   // between the kernels (tracing == 1) or MS_PDL=0
   const bool pdl = p->pdl && p->tracing != 1;
+  if (use_ranged(p, g.L) && p->one && p->k3v && p->kkind != IDS) {  // ONE cooperative launch (K3 v2 ONE mode)
+    uint32_t *HC = (uint32_t *)(w + g.off_hc);
+    const RangeScan rs{HC, offsets, 0, 1};
+    if (ev && p->tracing == 1) {
+      cudaEventRecord(ev[1], s);
+      cudaEventRecord(ev[2], s);
+    }
+    if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 2, nullptr, 0,
+                    &rs) != cudaSuccess)
+      return MS_ERR_CUDA;
+    if (ev) cudaEventRecord(ev[3], s);
+    p->last_launches = 1;
+    return MS_OK;
+  }
   if (use_ranged(p, g.L)) {  // K1r -> K2r -> K3 over C contiguous tile ranges (ms_ranged.cuh)
     uint32_t C = 0;
     if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 1, &C) != cudaSuccess ||

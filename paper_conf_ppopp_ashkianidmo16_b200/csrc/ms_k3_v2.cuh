@@ -30,6 +30,8 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
+#include <cooperative_groups.h>
+
 #include <type_traits>
 
 #include "ms_k3p_args.h"
@@ -61,7 +63,8 @@ struct K3vLayout {
   static constexpr int O_CNT = O_VS + (KV ? KSR * 4 : 0); // counters
   static constexpr int O_META = O_CNT + CNTB;             // [2][MW] words (tile parity)
   static constexpr int O_WS = O_META + 2 * MW * 4;        // warp sums [16]
-  static constexpr int O_BAR = (O_WS + 16 * 4 + 7) & ~7;  // mbarriers: keys [STAGES], values [STAGES]
+  static constexpr int O_TOT = O_WS + 16 * 4;             // ONE: this range's bucket totals [32]
+  static constexpr int O_BAR = (O_TOT + 32 * 4 + 7) & ~7; // mbarriers: keys [STAGES], values [STAGES]
   static constexpr int O_SPL = O_BAR + 2 * STAGES * 8;    // SPLITTERS: padded splitters [256] + bin table
   static constexpr int O_TBL = O_SPL + kMaxM * 4;
   static constexpr int BYTES = O_SPL;                     // + 1024 alignment slack at launch
@@ -77,7 +80,13 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *tm, in
       : "memory");
 }
 
-template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB, int KPT>
+// ONE (implies RANGED): the whole multisplit in ONE cooperative launch.  Phase 1
+// counts this CTA's range (K1r's job) through the same TMA pipeline, the range
+// counts are published to rs.HC, a grid-wide barrier, the range scan
+// (range_base) -- then phase 2 walks the range's tiles in REVERSE (the first
+// tiles it reads are the ones phase 1 read last, still in L2), with the running
+// G counting down from the range's end.
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB, int KPT, bool ONE = false>
 __global__ void __launch_bounds__(NT, MINB)
 k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv,
              const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
@@ -120,14 +129,28 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   const uint32_t ks32 = smem_u32(keys_s), vs32 = smem_u32(vals_s);
 
   const uint64_t r0 = RANGED ? (uint64_t)blockIdx.x * L / gridDim.x : 0;
-  auto tile_of = [&](uint32_t it) -> uint64_t {
-    return RANGED ? r0 + it : (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x;
-  };
   const uint32_t iters = RANGED ? (uint32_t)((uint64_t)(blockIdx.x + 1) * L / gridDim.x - r0)
                                 : (blockIdx.x < L ? (L - 1 - blockIdx.x) / gridDim.x + 1 : 0);
+  auto tile_of = [&](uint32_t it) -> uint64_t {
+    if constexpr (ONE) return r0 + iters - 1 - it;  // phase 2: reverse walk
+    return RANGED ? r0 + it : (uint64_t)blockIdx.x + (uint64_t)it * gridDim.x;
+  };
   const uint64_t Lfull = n / T;  // tiles the TMA loads; a partial last tile is loaded by hand
-  auto issue = [&](uint32_t it, bool values) {  // one thread: TMA of tile `it` into its stage
-    const uint64_t tile = tile_of(it);
+  // ONE: full tiles of the range, and whether the range ends with the partial tile
+  const uint32_t nf = ONE ? (uint32_t)(umin64(r0 + iters, Lfull) > r0 ? umin64(r0 + iters, Lfull) - r0 : 0) : 0;
+  const uint32_t ptail = ONE ? iters - nf : 0;  // 0 or 1
+  // TMA sequence numbers: ONE keys: phase 1 forward over the nf full tiles, then
+  // phase 2 reverse; ONE values: phase 2 only.  Otherwise sequence = iteration.
+  auto seq_tile = [&](uint32_t sq, bool values) -> uint64_t {
+    if constexpr (ONE) {
+      if (!values && sq < nf) return r0 + sq;
+      const uint32_t j = values ? sq : sq - nf;
+      return r0 + nf - 1 - j;
+    }
+    return tile_of(sq);
+  };
+  auto issue = [&](uint32_t it, bool values) {  // one thread: TMA of sequence `it` into its stage
+    const uint64_t tile = seq_tile(it, values);
     if (tile >= Lfull) return;
     const int st = (int)(it % STAGES);
     if (!values) {
@@ -146,9 +169,12 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       mbar_init(bar_v + s, 1);
     }
     fence_mbar_init();
-    for (uint32_t s = 0; s < (uint32_t)STAGES && s < iters; ++s) {
-      issue(s, false);
-      if constexpr (KV) issue(s, true);
+    const uint32_t nk = ONE ? 2 * nf : iters, nv = ONE ? nf : iters;
+    for (uint32_t s = 0; s < (uint32_t)STAGES; ++s) {
+      if (s < nk) issue(s, false);
+      if constexpr (KV) {
+        if (s < nv) issue(s, true);
+      }
     }
   }
   if constexpr (KIND == SPLITTERS) {
@@ -165,7 +191,69 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   uint32_t gnext = 0;  // tile mode: the next tile's G column
   uint32_t grun = 0;   // RANGED: G_row of the current tile (all threads of bucket row `row`)
   const uint32_t row = tid >> (LOGNT - LOGMP);
-  if constexpr (RANGED) {
+  uint32_t *tot_s = reinterpret_cast<uint32_t *>(sm + Ly::O_TOT);
+  if constexpr (ONE) {
+    // ---- phase 1: this range's bucket counts (private u16 counter columns,
+    // folded into tot_s every 2048 tiles so that no counter exceeds 32768)
+    if (tid < 32) tot_s[tid] = 0;
+    auto zero_cnt = [&]() {
+      uint4 *c4 = reinterpret_cast<uint4 *>(cnt);
+      for (int idx = tid; idx < Ly::CNTB / 16; idx += NT) c4[idx] = make_uint4(0, 0, 0, 0);
+    };
+    auto fold = [&]() {  // row sums of the counter matrix -> tot_s (then zero it)
+      __syncthreads();
+      constexpr uint32_t SEGS1 = NT >> LOGMP;  // threads per row, each 2*MP... plain bytes
+      constexpr uint32_t BPT = 2 * NT / SEGS1;  // bytes of a row per thread (= 2 * MP)
+      const uint32_t rr = tid / SEGS1, q = BPT * (tid % SEGS1);
+      uint32_t sum = 0;
+      for (uint32_t bq = 0; bq < BPT; bq += 4) {
+        const uint32_t o = q + bq;
+        sum = __dp2a_lo(*reinterpret_cast<const uint32_t *>(cnt + rr * RS + o + 16 * (o >> 7)), 0x0101u, sum);
+      }
+      if (rr < m && sum) atomicAdd(tot_s + rr, sum);
+      __syncthreads();
+      zero_cnt();
+      __syncthreads();
+    };
+    zero_cnt();
+    __syncthreads();
+    auto count1 = [&](uint32_t key) {
+      const uint32_t a = ccol + id_of(key) * RS;
+      sts_u16(a, lds_u16(a) + 1);
+    };
+    for (uint32_t sq = 0; sq < nf; ++sq) {
+      mbar_wait(bar_k + sq % STAGES, (sq / STAGES) & 1u);
+      const uint8_t *sk = sm + Ly::O_SK + (sq % STAGES) * TB;
+      uint4 kx[NCH];
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) kx[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) {
+        count1(kx[c].x); count1(kx[c].y); count1(kx[c].z); count1(kx[c].w);
+      }
+      // the stage may be refilled only once every thread's loads of it have
+      // RETURNED (values consumed above), not merely been issued
+      __syncthreads();
+      if (tid == 0 && sq + STAGES < 2 * nf) issue(sq + STAGES, false);
+      if ((sq & 2047u) == 2047u) fold();
+    }
+    if (ptail) {  // the partial last tile of the input
+      const uint64_t base = (r0 + nf) * T;
+      const uint32_t nt = (uint32_t)(n - base);
+      for (uint32_t q = 0; q < (uint32_t)K; ++q)
+        if (b0 + q < nt) count1(__ldg(keys + base + b0 + q));
+    }
+    fold();
+    if (tid < m) const_cast<uint32_t *>(rs.HC)[(uint64_t)blockIdx.x * m + tid] = tot_s[tid];
+    __threadfence();
+    cooperative_groups::this_grid().sync();
+    RangeScan r1 = rs;  // one row per CTA range
+    r1.R = gridDim.x;
+    r1.k = 1;
+    grun = range_base<NT, LOGMP>(r1, m, blockIdx.x, n, keys_s, row);
+    if (row < m) grun += tot_s[row];  // the reverse walk counts down from the range's end
+    __syncthreads();
+  } else if constexpr (RANGED) {
     if (rs.HC != nullptr) {  // K2r folded in: this range's G from K1r's rows (keys_s is free until tile 0)
       grun = range_base<NT, LOGMP>(rs, m, blockIdx.x, n, keys_s, row);
       __syncthreads();
@@ -183,8 +271,13 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     const uint64_t tile = tile_of(it);
     const uint64_t base = tile * T;
     const uint32_t nt = FULL ? (uint32_t)T : (uint32_t)(n - base);
-    const int st = (int)(it % STAGES);
-    const uint32_t ph = (it / STAGES) & 1u;
+    // key / value TMA sequence numbers of this tile (ONE: phase 1 used keys 0..nf-1;
+    // a partial tile, processed first in the reverse walk, has none)
+    const uint32_t kq = ONE ? nf + it - ptail : it, vq = ONE ? it - ptail : it;
+    const int st = (int)(kq % STAGES);
+    const uint32_t ph = (kq / STAGES) & 1u;
+    const int vst = (int)(vq % STAGES);
+    const uint32_t vph = (vq / STAGES) & 1u;
     uint32_t *meta = reinterpret_cast<uint32_t *>(sm + Ly::O_META) + (it & 1) * Ly::MW;
     uint32_t *rowS = meta;          // [MP+4]
     uint32_t *Pj = meta + MP + 4;   // [MP]
@@ -242,7 +335,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     }
     __syncthreads();
     // the key stage is free again (keys are in registers): refill it
-    if (tid == 0 && it + STAGES < iters) issue(it + STAGES, false);
+    if (FULL && tid == 0 && kq + STAGES < (ONE ? 2 * nf : iters)) issue(kq + STAGES, false);
 
     // ---- 2. CTA exclusive scan of the row-vectorised counter matrix:
     // thread t owns plain words [t*WPT, (t+1)*WPT) (inside one bucket row)
@@ -294,7 +387,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     if (tid == 0) rowS[MP] = tot;
     uint32_t Gr;
     if constexpr (RANGED) {
-      Gr = grun;
+      if constexpr (!ONE) Gr = grun;
       uint32_t rtot;  // this tile's count of bucket `row`
       if constexpr (TPR < 32) {
         rtot = __shfl_sync(0xFFFFFFFFu, excl + s, lane | (TPR - 1)) - Sr;
@@ -304,7 +397,12 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 #pragma unroll
         for (int i = 0; i < NW; ++i) rtot += ((uint32_t)i >= w0 && (uint32_t)i < w0 + TPR / 32) ? wsum[i] : 0u;
       }
-      grun += rtot;
+      if constexpr (ONE) {
+        grun -= rtot;
+        Gr = grun;
+      } else {
+        grun += rtot;
+      }
       if ((tid & (TPR - 1)) == 0) Gj[row] = Gr;
     } else {
       Gr = row < m ? Gj[row] : 0u;  // (fused sharded scatter: replaced by the destination offset below)
@@ -344,8 +442,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     uint4 vy[KV ? NCH : 1];
     if constexpr (KV) {
       if constexpr (FULL) {
-        mbar_wait(bar_v + st, ph);
-        const uint8_t *sv = sm + Ly::O_SV + st * TB;
+        mbar_wait(bar_v + vst, vph);
+        const uint8_t *sv = sm + Ly::O_SV + vst * TB;
 #pragma unroll
         for (int c = 0; c < NCH; ++c) vy[c] = *reinterpret_cast<const uint4 *>(sv + choff[c]);
       } else {
@@ -383,7 +481,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA (async proxy)
     __syncthreads();
     if constexpr (KV) {  // the value stage is free again: refill it
-      if (tid == 0 && it + STAGES < iters) issue(it + STAGES, true);
+      if (FULL && tid == 0 && vq + STAGES < (ONE ? nf : iters)) issue(vq + STAGES, true);
     }
 
     // ---- 4. bucket runs: SPB threads per bucket share its <= 3 head keys,
@@ -467,10 +565,15 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       }
     }
   };
-  const bool has_tail = iters && tile_of(iters - 1) >= Lfull;
-  const uint32_t iters_full = iters - (has_tail ? 1u : 0u);
-  for (uint32_t it = 0; it < iters_full; ++it) tile_body(it, std::true_type{});
-  if (has_tail) tile_body(iters_full, std::false_type{});
+  if constexpr (ONE) {  // reverse walk: the partial tile (if any) comes first
+    if (ptail) tile_body(0u, std::false_type{});
+    for (uint32_t it = ptail; it < iters; ++it) tile_body(it, std::true_type{});
+  } else {
+    const bool has_tail = iters && tile_of(iters - 1) >= Lfull;
+    const uint32_t iters_full = iters - (has_tail ? 1u : 0u);
+    for (uint32_t it = 0; it < iters_full; ++it) tile_body(it, std::true_type{});
+    if (has_tail) tile_body(iters_full, std::false_type{});
+  }
   if (ds.P > 0) bulk_wait0();  // peer stores complete before the grid ends (made visible by the stream order)
   else bulk_wait_read0();
 }
@@ -503,13 +606,13 @@ inline bool make_tile_map(CUtensorMap *tm, const uint32_t *ptr, uint64_t rows, u
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED>
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ONE = false>
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   // NT = 128 runs 32 keys per thread (same 4096-key tile, half the counter matrix per key)
   constexpr int KPT = NT == 128 ? 32 : 16;
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
   constexpr int MINB = NT == 256 ? (KV ? 2 : 3) : (KV ? 3 : 4);
-  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT>;
+  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
@@ -526,15 +629,20 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   CUtensorMap tmk, tmv;
   if (!make_tile_map(&tmk, a.keys, rows, Ly::T) || !make_tile_map(&tmv, KV ? a.vals : nullptr, rows, Ly::T))
     return cudaErrorInvalidValue;
-  const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals,
-                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs,
-                                  a.ds ? *a.ds : DistTarget{});
+  const cudaError_t e = ONE ? launch_coop(k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals, a.G,
+                                          a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs, DistTarget{})
+                            : launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys,
+                                        a.vals, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs,
+                                        a.ds ? *a.ds : DistTarget{});
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 template <int KIND, bool KV, int LOGMP, int NT>
 inline cudaError_t k3v_launch_n(const K3pArgs &a) {
   constexpr int STAGES = KV ? 1 : 2;
+  if constexpr (NT == 256) {
+    if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true>(a);
+  }
   return a.ranged ? k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true>(a)
                   : k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false>(a);
 }

@@ -45,7 +45,7 @@ struct K3pArgs {
   const BucketParams *bp;  // host copy, passed by value to the kernel
   int sms;
   cudaStream_t stream;
-  int ranged = 0;               // 1: CTA-range mode (G = GB[C][m], ms_ranged.cuh); m <= 32 only
+  int ranged = 0;               // 1: CTA-range mode (G = GB[C][m], ms_ranged.cuh); 2: one cooperative launch; m <= 32
   int pdl = 0;                  // 1: programmatic dependent launch after K2 (ms_device.cuh pdl_wait)
   uint32_t *grid_out = nullptr;  // non-null: only compute the grid C (no launch)
   RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged: fold K2r into K3's prologue when rs.HC is set
@@ -123,6 +123,23 @@ __device__ __forceinline__ uint32_t range_base(const RangeScan &rs, uint32_t m, 
   return row < m ? red[NT + row] : 0u;
 }
 
+
+// Cooperative launch (all CTAs co-resident; grid-wide barrier inside the kernel).
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_coop(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                               Args &&...args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 constexpr uint32_t kMaxRanges = 1024;  // upper bound on the CTA-range count C (workspace sizing)
 
