@@ -34,7 +34,7 @@ struct ms_plan_s {
   // 32 < m <= 256, kinds other than MS_IDS: MS_K3H=1 selects the two-digit K3
   // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
   int k3h = 0;
-  int one = 0;       // ranged variant as ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk)
+  int one = 1;       // ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk); MS_ONE=0 disables
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
   int32_t last_launches;
@@ -583,7 +583,11 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   // K2 and K3 use programmatic dependent launch unless per-stage events sit
   // between the kernels (tracing == 1) or MS_PDL=0
   const bool pdl = p->pdl && p->tracing != 1;
-  if (use_ranged(p, g.L) && p->one && p->k3v && p->kkind != IDS) {  // ONE cooperative launch (K3 v2 ONE mode)
+  // ONE cooperative launch (K3 v2 ONE mode), measured: key-only runs of the ranged
+  // variant, and key-only runs too small for it (L < 8 tiles per SM: 3 launches -> 1)
+  const bool one = p->one && p->k3v && p->kkind != IDS && p->spec.m <= 32 && !vals_in &&
+                   (p->flags & MS_VARIANT_3K) == 0 && (use_ranged(p, g.L) || g.L < 8ull * (uint64_t)sm_count());
+  if (one) {
     uint32_t *HC = (uint32_t *)(w + g.off_hc);
     const RangeScan rs{HC, offsets, 0, 1};
     if (ev && p->tracing == 1) {

@@ -14,6 +14,6 @@ for nm in names:
     r = bench.bench_config(nm, bench.CONFIGS[nm], steps, 3, torch.device("cuda"), 1, 0, with_e2e=False)
     st = r["stages_ms"]
     print(f"{tag} {nm:6s} {r['value']:8.2f} Gk/s  step {r['ms_per_step']:.4f} ms  whole {r['whole_step_frac']:.3f}  "
-          f"K1 {st['k1_prescan']:.4f} ({r['roofline']['k1_prescan_frac']:.3f})  K2 {st['k2_scan']:.4f}  "
+          f"K1 {st['k1_prescan']:.4f} ({r['roofline']['k1_prescan_frac'] or 0:.3f})  K2 {st['k2_scan']:.4f}  "
           f"K3 {st['k3_postscan']:.4f} ({r['roofline']['frac']:.3f})  nopdl {st['sum_without_pdl']:.4f}  "
-          f"T={r['tile']} v={r['variant']}", flush=True)
+          f"T={r['tile']} v={r['variant']} launches={r['gpu_launches'] // steps}", flush=True)
