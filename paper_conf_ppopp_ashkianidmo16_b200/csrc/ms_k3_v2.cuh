@@ -98,7 +98,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   constexpr int NW = NT / 32;
   constexpr int NCH = K / 4;  // 16-byte chunks per thread block
   constexpr int LOGNT = NT == 256 ? 8 : 7;
-  constexpr bool KEEP_ID = KIND == SPLITTERS;  // the table lookup is kept, not repeated
+  constexpr bool KEEP_ID = KIND == SPLITTERS || KIND == DELTA;  // multi-instruction ids are kept, not recomputed
   extern __shared__ uint8_t smraw[];
   // align to 1024 B by offsetting the shared pointer itself (an integer round
   // trip would turn every access below into a generic LD/ST)
