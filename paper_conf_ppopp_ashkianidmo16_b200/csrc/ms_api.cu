@@ -34,6 +34,7 @@ struct ms_plan_s {
   // 32 < m <= 256, kinds other than MS_IDS: MS_K3H=1 selects the two-digit K3
   // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
   int k3h = 0;
+  int tile_forced = 0;  // MS_VARIANT_3K flag or MS_VARIANT=tile
   int one = 1;       // ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk); MS_ONE=0 disables
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
@@ -391,6 +392,9 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
     if (strcmp(e, "ranged") == 0 && m <= 32) p->ranged = 2;
   }
   if (flags & MS_VARIANT_3K) p->ranged = 0;
+  p->tile_forced = (flags & MS_VARIANT_3K) ? 1 : 0;
+  if (const char *e = getenv("MS_VARIANT"))
+    if (strcmp(e, "tile") == 0) p->tile_forced = 1;
   if (flags & MS_VARIANT_RANGED) p->ranged = 2;
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
@@ -585,8 +589,9 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   const bool pdl = p->pdl && p->tracing != 1;
   // ONE cooperative launch (K3 v2 ONE mode), measured: key-only runs of the ranged
   // variant, and key-only runs too small for it (L < 8 tiles per SM: 3 launches -> 1)
-  const bool one = p->one && p->k3v && p->kkind != IDS && p->spec.m <= 32 && !vals_in &&
-                   (p->flags & MS_VARIANT_3K) == 0 && (use_ranged(p, g.L) || g.L < 8ull * (uint64_t)sm_count());
+  // (m <= 32 key-only: ONE beats the 3-kernel tile variant too -- NSko 410 -> 422 G keys/s -- unless
+  // the tile variant is forced by MS_VARIANT_3K / MS_VARIANT=tile)
+  const bool one = p->one && p->k3v && p->kkind != IDS && p->spec.m <= 32 && !vals_in && !p->tile_forced;
   if (one) {
     uint32_t *HC = (uint32_t *)(w + g.off_hc);
     const RangeScan rs{HC, offsets, 0, 1};
