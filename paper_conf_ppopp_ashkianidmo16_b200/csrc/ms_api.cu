@@ -35,6 +35,7 @@ struct ms_plan_s {
   // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
   int k3h = 0;
   int tile_forced = 0;  // MS_VARIANT_3K flag or MS_VARIANT=tile
+  int direct = 0;       // ablation MS_K3_DIRECT=1: K3 stores keys straight to global, no local reorder
   int one = 1;       // ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk); MS_ONE=0 disables
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
@@ -200,6 +201,7 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   a.ranged = ranged;
   a.grid_out = grid_out;
   a.pdl = pdl;
+  a.direct = p->direct;
   if (rs) a.rs = *rs;
   if (p->spec.m <= 32 && p->k3v && p->kkind != IDS) {  // K3 v2 (ms_k3_v2.cuh)
     switch (p->kkind) {
@@ -395,6 +397,13 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->tile_forced = (flags & MS_VARIANT_3K) ? 1 : 0;
   if (const char *e = getenv("MS_VARIANT"))
     if (strcmp(e, "tile") == 0) p->tile_forced = 1;
+  if (const char *e = getenv("MS_K3_DIRECT")) {
+    p->direct = atoi(e) ? 1 : 0;
+    if (p->direct) {
+      p->tile_forced = 1;  // the ablation runs the 3-kernel tile variant
+      p->ranged = 0;
+    }
+  }
   if (flags & MS_VARIANT_RANGED) p->ranged = 2;
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;

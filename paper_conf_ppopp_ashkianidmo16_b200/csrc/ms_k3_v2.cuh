@@ -45,7 +45,7 @@ struct K3vLayout {
   static constexpr int T = NT * K;              // keys per tile
   static constexpr int TB = T * 4;              // bytes of one staged array (keys or values)
   static constexpr int KSR = (T + 3 * MP + 4 + 3) & ~3;  // reorder slots incl. alignment padding
-  static constexpr int MW = 3 * MP + 8;         // per-tile metadata words: rowS[MP+4] P[MP] G[MP]
+  static constexpr int MW = 4 * MP + 8;         // per-tile metadata words: rowS[MP+4] P[MP] G[MP] D[MP]
   // u16 counter matrix c[j][beta], row-major; inside a row, 16 bytes of
   // padding after every 128 bytes (byte q of a plain row lives at
   // q + 16 * (q / 128)), and the row stride is rounded up to a multiple of
@@ -86,7 +86,10 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *tm, in
 // (range_base) -- then phase 2 walks the range's tiles in REVERSE (the first
 // tiles it reads are the ones phase 1 read last, still in L2), with the running
 // G counting down from the range's end.
-template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB, int KPT, bool ONE = false>
+// DIRECT (ablation, SURVEY NEXT-2 / the paper's "Direct" method of Table 4): no local reorder --
+// every key is stored from registers straight to its global position G_j + local offset.
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB, int KPT, bool ONE = false,
+          bool DIRECT = false>
 __global__ void __launch_bounds__(NT, MINB)
 k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv,
              const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
@@ -282,6 +285,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     uint32_t *rowS = meta;          // [MP+4]
     uint32_t *Pj = meta + MP + 4;   // [MP]
     uint32_t *Gj = Pj + MP;         // [MP]
+    uint32_t *Dj = Gj + MP;         // [MP] DIRECT: G_j - P_j
 
     // ---- 0. zero the counters (last read by the previous tile's scatter,
     // before its final barrier); publish this tile's G column
@@ -435,6 +439,9 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       else *reinterpret_cast<uint32_t *>(dst) = w[i][0];
     }
     if ((tid & (TPR - 1)) == 0) Pj[row] = Sr + pad;
+    if constexpr (DIRECT) {
+      if ((tid & (TPR - 1)) == 0) Dj[row] = Gr - (Sr + pad);
+    }
     bulk_wait_read0();  // this thread's bulk stores of the previous tile have read keys_s/vals_s
     __syncthreads();
 
@@ -461,20 +468,27 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       if constexpr (KV) {
         vv[0] = vy[c].x; vv[1] = vy[c].y; vv[2] = vy[c].z; vv[3] = vy[c].w;
       }
-      uint32_t sl[4];
+      uint32_t sl[4], idv[4];
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         uint32_t id;
         if constexpr (KEEP_ID) id = __byte_perm(idk[c], 0u, 0x4440u + j);
         else id = id_of(kk[j]);
+        idv[j] = id;
         sl[j] = (FULL || b0 + 4 * c + j < nt) ? lds_u16(ccol + id * RS) : 0u;
       }
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         if (FULL || b0 + 4 * c + j < nt) {
           const uint32_t slot = sl[j] + __byte_perm(rk[c], 0u, 0x4440u + j);
-          sts_u32(ks32 + 4 * slot, kk[j]);
-          if constexpr (KV) sts_u32(vs32 + 4 * slot, vv[j]);
+          if constexpr (DIRECT) {
+            const uint32_t dst = Dj[idv[j]] + slot;
+            keys_out[dst] = kk[j];
+            if constexpr (KV) vals_out[dst] = vv[j];
+          } else {
+            sts_u32(ks32 + 4 * slot, kk[j]);
+            if constexpr (KV) sts_u32(vs32 + 4 * slot, vv[j]);
+          }
         }
       }
     }
@@ -486,7 +500,9 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 
     // ---- 4. bucket runs: SPB threads per bucket share its <= 3 head keys,
     // <= 3 tail keys and the TMA bulk store(s) of the 16-byte-aligned body
-    if (!RANGED && ds.P > 0) {
+    if (DIRECT) {
+      // (stored in step 3)
+    } else if (!RANGED && ds.P > 0) {
       // fused sharded scatter: the run [gs, gs + len) of global positions is
       // cut at window boundaries; each piece goes to its owner's window, the
       // 16-byte-aligned body by one TMA bulk store per array (peer memory is
@@ -606,13 +622,13 @@ inline bool make_tile_map(CUtensorMap *tm, const uint32_t *ptr, uint64_t rows, u
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ONE = false>
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ONE = false, bool DIRECT = false>
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   // NT = 128 runs 32 keys per thread (same 4096-key tile, half the counter matrix per key)
   constexpr int KPT = NT == 128 ? 32 : 16;
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
   constexpr int MINB = NT == 256 ? (KV ? 2 : 3) : (KV ? 3 : 4);
-  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE>;
+  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE, DIRECT>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
@@ -642,6 +658,10 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
   constexpr int STAGES = KV ? 1 : 2;
   if constexpr (NT == 256) {
     if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true>(a);
+  }
+  if (a.direct) {  // ablation: instantiated for the one-shift bucket kind only (SHIFT: DELTA with m*delta = 2^32)
+    if constexpr (NT == 256 && KIND == SHIFT) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, true>(a);
+    return cudaErrorNotSupported;
   }
   return a.ranged ? k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true>(a)
                   : k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false>(a);

@@ -50,6 +50,7 @@ struct K3pArgs {
   uint32_t *grid_out = nullptr;  // non-null: only compute the grid C (no launch)
   RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged: fold K2r into K3's prologue when rs.HC is set
   const DistTarget *ds = nullptr;           // fused sharded scatter (K3 v2, tile variant only)
+  int direct = 0;                           // ablation: K3 v2 without the local reorder (MS_K3_DIRECT=1)
 };
 
 // Launch with cudaLaunchAttributeProgrammaticStreamSerialization when `pdl`:

@@ -381,3 +381,15 @@ def test_fused_scatter_rejects_unsupported():
         with pytest.raises(_abi.MultisplitError) as e:
             plan.postscan_scatter(keys, G, t)
         assert e.value.status == _abi.MS_ERR_UNSUPPORTED
+
+
+@pytest.mark.parametrize("m", [2, 8, 32])
+def test_parity_direct_ablation(m, monkeypatch):
+    """The Direct (no local reorder) K3 ablation, MS_K3_DIRECT=1 (SHIFT bucket kind: DELTA with
+    m * delta = 2^32), bit-exact on ragged sizes, KO and KV."""
+    monkeypatch.setenv("MS_K3_DIRECT", "1")
+    for i, n in enumerate([1, 4095, 4097, 100003, (1 << 21) + 3]):
+        for kv in (False, True):
+            case = make_case("delta", m, n, seed=2 * (400 + i), kv=kv)  # even seed: delta = 2^32 / m
+            assert case["spec_kw"]["delta"] == (1 << 32) // m
+            _assert_equal(case, _run_case(case), _expect(case), f"direct m={m} n={n} kv={kv}")
