@@ -35,6 +35,7 @@ struct ms_plan_s {
   // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
   int k3h = 0;
   int tile_forced = 0;  // MS_VARIANT_3K flag or MS_VARIANT=tile
+  uint32_t k1s_per_sm = 8;  // splitter K1: persistent CTAs per SM (each builds the bin table once; MS_K1S_PER_SM)
   int direct = 0;       // ablation MS_K3_DIRECT=1: K3 stores keys straight to global, no local reorder
   int one = 1;       // ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk); MS_ONE=0 disables
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
@@ -165,7 +166,7 @@ cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *key
                                  : k1_prescan<KIND, KPT, SUBT>;                                     \
     set_smem(k, smem);                                                                             \
     uint64_t grid = (g.L + SUBT - 1) / SUBT;                                                       \
-    if (KIND == SPLITTERS && p->spec.m <= 32) grid = std::min<uint64_t>(grid, 8ull * (uint64_t)sm_count()); \
+    if (KIND == SPLITTERS && p->spec.m <= 32) grid = std::min<uint64_t>(grid, (uint64_t)p->k1s_per_sm * sm_count()); \
     k<<<(unsigned)grid, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, zero_words, \
                                              flag);                                                \
   }
@@ -397,6 +398,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->tile_forced = (flags & MS_VARIANT_3K) ? 1 : 0;
   if (const char *e = getenv("MS_VARIANT"))
     if (strcmp(e, "tile") == 0) p->tile_forced = 1;
+  if (const char *e = getenv("MS_K1S_PER_SM")) p->k1s_per_sm = std::max(1, std::min(16, atoi(e)));
   if (const char *e = getenv("MS_K3_DIRECT")) {
     p->direct = atoi(e) ? 1 : 0;
     if (p->direct) {
