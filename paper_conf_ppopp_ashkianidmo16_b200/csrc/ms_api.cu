@@ -37,6 +37,7 @@ struct ms_plan_s {
   int tile_forced = 0;  // MS_VARIANT_3K flag or MS_VARIANT=tile
   uint32_t k1s_per_sm = 8;  // splitter K1: persistent CTAs per SM (each builds the bin table once; MS_K1S_PER_SM)
   int direct = 0;       // ablation MS_K3_DIRECT=1: K3 stores keys straight to global, no local reorder
+  int one_kv = 1;    // ONE for key-value runs: 0 never, 1 when L <= 64 tiles per SM, 2 always (MS_ONE_KV)
   int one = 1;       // ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk); MS_ONE=0 disables
   int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
   int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
@@ -410,6 +411,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_ONE")) p->one = atoi(e) ? 1 : 0;
+  if (const char *e = getenv("MS_ONE_KV")) p->one_kv = std::max(0, std::min(2, atoi(e)));
   if (const char *e = getenv("MS_K3H")) p->k3h = atoi(e) ? 1 : 0;
   if (const char *e = getenv("MS_RANGED_K2")) p->fuse_k2r = atoi(e) ? 0 : 1;
   *plan = p;
@@ -602,7 +604,10 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   // variant, and key-only runs too small for it (L < 8 tiles per SM: 3 launches -> 1)
   // (m <= 32 key-only: ONE beats the 3-kernel tile variant too -- NSko 410 -> 422 G keys/s -- unless
   // the tile variant is forced by MS_VARIANT_3K / MS_VARIANT=tile)
-  const bool one = p->one && p->k3v && p->kkind != IDS && p->spec.m <= 32 && !vals_in && !p->tile_forced;
+  // key-value: ONE at up to 64 tiles per SM (C3, n = 2^25: 192 -> 207 G keys/s), not above
+  // (NSkv, n = 2^28: 293 -> 276 -- the two/three-launch paths stream better there)
+  const bool one = p->one && p->k3v && p->kkind != IDS && p->spec.m <= 32 && !p->tile_forced &&
+                   (!vals_in || p->one_kv == 2 || (p->one_kv == 1 && g.L <= 64ull * (uint64_t)sm_count()));
   if (one) {
     uint32_t *HC = (uint32_t *)(w + g.off_hc);
     const RangeScan rs{HC, offsets, 0, 1};

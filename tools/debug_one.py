@@ -22,7 +22,8 @@ C = min(L, 444)
 ids_np = np.asarray(oracle.bucket_ids(case["ospec"], case["keys"]) if hasattr(oracle, "bucket_ids") else None)
 for rep in range(int(os.environ.get("REPS", "1"))):
     ko = torch.empty_like(kd)
-    plan.run(kd, vd, keys_out=ko, vals_out=(torch.empty_like(vd) if vd is not None else None), workspace=ws)
+    vo = torch.empty_like(vd) if vd is not None else None
+    plan.run(kd, vd, keys_out=ko, vals_out=vo, workspace=ws)
     torch.cuda.synchronize()
     if not np.array_equal(from_dev(ko), eko0):
         fails += 1
