@@ -72,9 +72,23 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
       uint32_t diff = FULL ? 0u : ~__ballot_sync(0xFFFFFFFFu, valid);
 #pragma unroll
       for (int b = 0; b < LOGM; ++b) {
-        const int32_t sh = (int32_t)(id << (31 - b));
-        const uint32_t vote = __ballot_sync(0xFFFFFFFFu, sh < 0);
-        diff |= vote ^ (uint32_t)(sh >> 31);
+        if constexpr (!KV) {
+          // 4 instructions per id bit: predicate from the bit (LOP3.P), ballot, predicated NOT,
+          // OR (measured: C4ko 213 -> 236 G keys/s, m64 KO 286 -> 340)
+          asm("{\n\t.reg .pred p;\n\t.reg .b32 t;\n\t"
+              "setp.ne.u32 p, %1, 0;\n\t"
+              "vote.sync.ballot.b32 t, p, 0xffffffff;\n\t"
+              "@p not.b32 t, t;\n\t"
+              "or.b32 %0, %0, t;\n\t}"
+              : "+r"(diff)
+              : "r"(id & (1u << b)));
+        } else {
+          // key-value: the compiler's 5-instruction form schedules better around the value
+          // registers (the inline form measured 10-15 % slower for KV)
+          const int32_t sh = (int32_t)(id << (31 - b));
+          const uint32_t vote = __ballot_sync(0xFFFFFFFFu, sh < 0);
+          diff |= vote ^ (uint32_t)(sh >> 31);
+        }
       }
       peers = ~diff;
     }
