@@ -15,14 +15,20 @@
  *   K2 scan       G = exclusive scan of row-vectorised H, offsets = G[:,0]
  *   K3 post-scan  recompute ids, stable tile-local multisplit in shared
  *                 memory, coalesced scatter to G[j][l] + local offset
- * Two variants (ms_plan_geometry reports which one a plan uses):
- *   0 "tile"   subproblems = the L tiles (H, G are m x L words);
- *   1 "ranged" (default for m <= 32) subproblems = the C <= 2048 contiguous
- *              tile ranges of K3's persistent CTAs: K1 writes per-range
- *              histograms (m x C), K2 is a one-CTA scan of them, and K3 keeps
- *              each tile's G_j as a running sum inside its range (Eq. (2)
- *              applied twice).
- * The stage-wise calls (ms_prescan / ms_scan / ms_postscan) always use tiles.
+ * Variants (ms_plan_geometry reports tile (0) or ranged (1); ms_plan_last_launches
+ * how many kernels the last ms_run enqueued):
+ *   "tile"   subproblems = the L tiles (H, G are m x L words): K1, K2, K3;
+ *   "ranged" subproblems = the C <= 1024 contiguous tile ranges of K3's
+ *            persistent CTAs: K1 writes per-range histograms (C x k x m), K3
+ *            folds their scan into its prologue and keeps each tile's G_j as a
+ *            running sum inside its range (Eq. (2) applied twice): 2 kernels;
+ *   "ONE"    (m <= 32, computed ids; every key-only run and key-value runs of
+ *            up to 64 tiles per SM) the ranged form in ONE cooperative launch:
+ *            range counts, grid barrier, range scan, post-scan (reverse tile
+ *            walk) -- 1 kernel.  DESIGN.md §7.
+ * Every variant computes the same (unique, stable) result.  MS_VARIANT_3K
+ * forces the tile variant.  The stage-wise calls (ms_prescan / ms_scan /
+ * ms_postscan) always use tiles.
  *
  * Conventions for every call below:
  *  - Pointers named *_in/*_out/ids/offsets/workspace/H/G are CUDA DEVICE
