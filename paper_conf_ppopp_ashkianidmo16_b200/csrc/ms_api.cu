@@ -615,12 +615,17 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
       cudaEventRecord(ev[1], s);
       cudaEventRecord(ev[2], s);
     }
-    if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 2, nullptr, 0,
-                    &rs) != cudaSuccess)
-      return MS_ERR_CUDA;
-    if (ev) cudaEventRecord(ev[3], s);
-    p->last_launches = 1;
-    return MS_OK;
+    const cudaError_t e1 = dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 2,
+                                       nullptr, 0, &rs);
+    if (e1 == cudaSuccess) {
+      if (ev) cudaEventRecord(ev[3], s);
+      p->last_launches = 1;
+      return MS_OK;
+    }
+    // the grid could not be made co-resident (e.g. the GPU is partitioned / shared): clear the
+    // launch error and take the multi-launch path below (same result)
+    if (e1 != cudaErrorCooperativeLaunchTooLarge) return MS_ERR_CUDA;
+    cudaGetLastError();
   }
   if (use_ranged(p, g.L)) {  // K1r -> K2r -> K3 over C contiguous tile ranges (ms_ranged.cuh)
     uint32_t C = 0;
