@@ -682,7 +682,7 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
 
 template <int KIND, bool KV, int LOGMP, int NT>
 inline cudaError_t k3v_launch_n(const K3pArgs &a) {
-  constexpr int STAGES = KV ? 1 : 2;
+  constexpr int STAGES = KV ? 1 : (LOGMP <= 3 && NT == 256 ? 3 : 2);  // m <= 8 key-only: 3 stages still fit 3 CTAs/SM
   if constexpr (NT == 256) {
     if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true>(a);
   }
