@@ -89,6 +89,62 @@ __device__ __forceinline__ uint32_t range_base(const RangeScan &rs, uint32_t m, 
   constexpr uint32_t MP = 1u << LOGMP, NS = NT / MP;
   const uint32_t tid = threadIdx.x, j = tid & (MP - 1), s = tid >> LOGMP;
   const uint32_t cut = c * rs.k;
+  if (MP >= 4 && m == MP) {
+    // m a power of two >= 4: 128-bit loads (thread t always reads column group t mod MP/4 of
+    // rows t/(MP/4), (t+NT)/(MP/4), ...), lane-shuffle reduction per warp, then the warps' partials
+    constexpr uint32_t Q4 = MP >= 4 ? MP / 4 : 1, NW = NT / 32;
+    const uint32_t lane = tid & 31, warp = tid >> 5, cg = tid & (Q4 - 1);
+    uint32_t pr[4] = {0u, 0u, 0u, 0u}, po[4] = {0u, 0u, 0u, 0u};
+    const uint4 *h4 = reinterpret_cast<const uint4 *>(rs.HC);
+    const uint32_t tot4 = rs.R * Q4;
+#pragma unroll 4
+    for (uint32_t u = tid; u < tot4; u += NT) {
+      const uint4 v = __ldcg(h4 + u);
+      const uint32_t vv[4] = {v.x, v.y, v.z, v.w};
+      const bool before = u / Q4 < cut;
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        pr[e] += before ? vv[e] : 0u;
+        po[e] += before ? 0u : vv[e];
+      }
+    }
+#pragma unroll
+    for (uint32_t off = 16; off >= Q4; off >>= 1) {
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        pr[e] += __shfl_xor_sync(0xFFFFFFFFu, pr[e], off);
+        po[e] += __shfl_xor_sync(0xFFFFFFFFu, po[e], off);
+      }
+    }
+    if (lane < Q4) {
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        red[warp * 32 + cg * 4 + e] = pr[e];
+        red[NT + warp * 32 + cg * 4 + e] = po[e];
+      }
+    }
+    __syncthreads();
+    uint32_t pj = 0, qj = 0;
+    if (tid < m) {
+#pragma unroll
+      for (uint32_t w = 0; w < NW; ++w) {
+        pj += red[w * 32 + tid];
+        qj += red[NT + w * 32 + tid];
+      }
+    }
+    __syncthreads();
+    if (tid < 32) {
+      const uint32_t tot = pj + qj;  // 0 for tid >= m
+      const uint32_t start = warp_incl_scan(tot, tid) - tot;
+      if (tid < m) red[NT + tid] = start + pj;
+      if (c == 0 && rs.offsets != nullptr) {
+        if (tid < m) rs.offsets[tid] = start;
+        if (tid == 0) rs.offsets[m] = n;
+      }
+    }
+    __syncthreads();
+    return row < m ? red[NT + row] : 0u;
+  }
   uint32_t pre = 0, post = 0;
   if (j < m) {
     const uint32_t *col = rs.HC + j;
