@@ -106,6 +106,37 @@ def test_run_argument_errors_without_gpu():
     L.ms_plan_destroy(h2)
 
 
+def test_postscan_scatter_argument_errors_without_gpu():
+    """ms_postscan_scatter (fused sharded scatter) refuses bad targets before touching CUDA."""
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import scatter_target
+    L = _abi.lib()
+    P = ctypes.c_void_p
+    A, B, W = P(0x10000000), P(0x20000000), P(0x30000000)
+    big = 1 << 20
+    st, h = _create(BucketSpec("delta", 8, delta=5), max_n=4096, kv=0)
+    t = scatter_target([0x40000000, 0x50000000], None, [0, 50, 100], [0] * 8)
+    call = lambda tg, n=100, k=A, g=B: L.ms_postscan_scatter(h, k, None, g, n, tg, W, big, None)
+    assert call(None) == _abi.MS_ERR_INVALID_ARG                                   # no target
+    assert call(ctypes.byref(t), k=None) == _abi.MS_ERR_INVALID_ARG                # null keys
+    assert call(ctypes.byref(t), g=P(0x20000004)) == _abi.MS_ERR_ALIGNMENT         # misaligned G
+    bad = scatter_target([0x40000000, 0], None, [0, 50, 100], [0] * 8)
+    assert call(ctypes.byref(bad)) == _abi.MS_ERR_INVALID_ARG                      # non-empty window, no pointer
+    bad = scatter_target([0x40000000, 0x50000004], None, [0, 50, 100], [0] * 8)
+    assert call(ctypes.byref(bad)) == _abi.MS_ERR_ALIGNMENT                        # misaligned window
+    bad = scatter_target([0x40000000, 0x50000000], None, [0, 60, 50], [0] * 8)
+    assert call(ctypes.byref(bad)) == _abi.MS_ERR_INVALID_ARG                      # decreasing window starts
+    t.nranks = 0
+    assert call(ctypes.byref(t)) == _abi.MS_ERR_INVALID_ARG
+    t.nranks = 9
+    assert call(ctypes.byref(t)) == _abi.MS_ERR_INVALID_ARG
+    L.ms_plan_destroy(h)
+    for spec in (BucketSpec("delta", 64, delta=5), BucketSpec("ids", 8, id_bytes=1)):
+        st, h = _create(spec, max_n=4096, kv=0)
+        t = scatter_target([0x40000000], None, [0, 100], [0] * 32)
+        assert L.ms_postscan_scatter(h, A, None, B, 100, ctypes.byref(t), W, big, None) == _abi.MS_ERR_UNSUPPORTED
+        L.ms_plan_destroy(h)
+
+
 def test_status_strings():
     for s in [0, -1, -2, -3, -4, -5, -6, -8]:
         assert _abi.status_string(s) and _abi.status_string(s) != "unknown status"
