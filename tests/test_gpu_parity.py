@@ -50,16 +50,16 @@ NS = [0, 1, 31, 2047, 2048, 2049, 4095, 4097, 8191, 8193, 100003]
 MS = [1, 2, 3, 5, 8, 31, 32, 33, 64, 127, 255, 256]
 
 
-@pytest.mark.parametrize("variant", [None, "ranged"])
-@pytest.mark.parametrize("kind", ["lowbits", "delta", "splitters", "ids"])
-@pytest.mark.parametrize("m", MS)
+# Low-bit buckets need a power-of-two m (reading #10); m > 32 always uses the tile variant, so the
+# forced CTA-range variant is only generated for m <= 32.
+MATRIX = [(kind, m, variant) for variant in (None, "ranged") for kind in ("lowbits", "delta", "splitters", "ids")
+          for m in MS if not (kind == "lowbits" and m & (m - 1)) and not (variant == "ranged" and m > 32)]
+
+
+@pytest.mark.parametrize("kind,m,variant", MATRIX)
 def test_parity_matrix(kind, m, variant):
     """kind x m x n (empty, ragged, tile edges) x KO/KV, uniform keys; the default
     variant (tile at these sizes) and the forced CTA-range variant (m <= 32)."""
-    if kind == "lowbits" and m & (m - 1):
-        pytest.skip("low-bit buckets need a power-of-two m (reading #10)")
-    if variant == "ranged" and m > 32:
-        pytest.skip("m > 32 always uses the tile variant")
     for i, n in enumerate(NS):
         for kv in (False, True):
             case = make_case(kind, m, n, seed=1000 * m + i, kv=kv, id_bytes=1 if i % 2 else 4)
@@ -87,13 +87,11 @@ def test_ranged_range_edges(kind, m, kv, k2r, monkeypatch):
             _assert_equal(case, _run_case(case, "ranged"), _expect(case), f"{kind} m={m} L={L} n={n}")
 
 
-@pytest.mark.parametrize("kind", ["lowbits", "delta", "splitters"])
-@pytest.mark.parametrize("m", [33, 64, 127, 256])
+@pytest.mark.parametrize("kind,m", [(k, m) for k in ("lowbits", "delta", "splitters") for m in (33, 64, 127, 256)
+                                    if not (k == "lowbits" and m & (m - 1))])
 def test_parity_two_digit_k3(kind, m, monkeypatch):
     """The two-digit (LSD 16 x 16) K3 for m > 32, an ablation kept behind MS_K3H=1: bit-exact on ragged
     sizes, skewed buckets and a multi-wave n."""
-    if kind == "lowbits" and m & (m - 1):
-        pytest.skip("low-bit buckets need a power-of-two m (reading #10)")
     monkeypatch.setenv("MS_K3H", "1")
     for i, (n, dist) in enumerate([(1, "uniform"), (4095, "uniform"), (4097, "hot"), (100003, "binomial"),
                                    ((1 << 22) + 5, "uniform")]):
