@@ -80,11 +80,16 @@ for f in sorted(os.listdir(src)):
     c = bench.CONFIGS[cfg]
     pre, post = model.pass_bytes_per_key(c["kv"])
     alg = (post if kern.startswith("k3") else pre if kern.startswith("k1") else 0) * c["n"]
+    # the library's ONE rule (ms_api.cu): m <= 32 key-only, or key-value up to 64
+    # tiles per SM, runs K1 + K3 in one cooperative k3v_postscan launch -> 12 / 20 B per key
+    one = kern == "k3v_postscan" and c["m"] <= 32 and (not c["kv"] or c["n"] // 4096 <= 64 * 148)
+    if one:
+        alg = (pre + post) * c["n"]
     stalls = [(hh.replace("smsp__average_warps_issue_stalled_", "").replace("_per_issue_active.ratio", ""),
                float(d[i] or 0)) for i, hh in enumerate(h)
               if hh.startswith("smsp__average_warps_issue_stalled_") and hh.endswith("_per_issue_active.ratio")]
     stalls.sort(key=lambda x: -x[1])
-    out.append(f"## {kern} on {cfg} ({c['desc']})\n")
+    out.append(f"## {kern}{' (ONE: K1 + K3 in one launch)' if one else ''} on {cfg} ({c['desc']})\n")
     out.append(f"- duration {t_us:.1f} us (under ncu, clocks not locked); dram read+write {dram / 1e9:.4f} GB"
                + (f" vs algorithmic {alg / 1e9:.4f} GB (ratio {dram / alg:.3f})" if alg else ""))
     for k in keys[3:]:
