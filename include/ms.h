@@ -15,19 +15,19 @@
  *   K2 scan       G = exclusive scan of row-vectorised H, offsets = G[:,0]
  *   K3 post-scan  recompute ids, stable tile-local multisplit in shared
  *                 memory, coalesced scatter to G[j][l] + local offset
- * Variants (ms_plan_geometry reports tile (0) or ranged (1); ms_plan_last_launches
- * how many kernels the last ms_run enqueued):
+ * Variants (ms_plan_geometry reports tile (0), ranged (1) or ONE (2);
+ * ms_plan_last_launches how many kernels the last ms_run enqueued):
  *   "tile"   subproblems = the L tiles (H, G are m x L words): K1, K2, K3;
  *   "ranged" subproblems = the C <= 1024 contiguous tile ranges of K3's
  *            persistent CTAs: K1 writes per-range histograms (C x k x m), K3
  *            folds their scan into its prologue and keeps each tile's G_j as a
  *            running sum inside its range (Eq. (2) applied twice): 2 kernels;
- *   "ONE"    (m <= 32, computed ids; every key-only run and key-value runs of
- *            up to 64 tiles per SM) the ranged form in ONE cooperative launch:
- *            range counts, grid barrier, range scan, post-scan (reverse tile
- *            walk) -- 1 kernel.  DESIGN.md §7.
- * Every variant computes the same (unique, stable) result.  MS_VARIANT_3K
- * forces the tile variant.  The stage-wise calls (ms_prescan / ms_scan /
+ *   "ONE"    (m <= 32; every key-only run and key-value runs of up to 64
+ *            tiles per SM) the ranged form in ONE cooperative launch: range
+ *            counts, grid barrier, range scan, post-scan (reverse tile walk)
+ *            -- 1 kernel.  DESIGN.md §7.
+ * Every variant computes the same (unique, stable) result.  The MS_VARIANT_*
+ * plan flags force one.  The stage-wise calls (ms_prescan / ms_scan /
  * ms_postscan) always use tiles.
  *
  * Conventions for every call below:
@@ -61,6 +61,7 @@ typedef int32_t ms_status;
 #define MS_ERR_ALIAS         (-4) /* an output overlaps an input                               */
 #define MS_ERR_WORKSPACE     (-5) /* workspace NULL or smaller than ms_plan_workspace_size()   */
 #define MS_ERR_CUDA          (-6) /* a CUDA runtime call failed                                */
+#define MS_ERR_NCCL          (-7) /* an NCCL call failed (ms_dist_run)                          */
 #define MS_ERR_BUCKET_RANGE  (-8) /* MS_VALIDATE: some precomputed id was >= m                 */
 
 /* Bucket identifier kinds: the programmer's whatBucket() (P:353-357,
@@ -86,23 +87,42 @@ typedef struct {
 
 typedef struct ms_plan_s *ms_plan_t;
 
-/* plan flags */
-#define MS_VALIDATE      1u  /* flag precomputed ids >= m on the device; ms_plan_check reports it */
-#define MS_VARIANT_3K     2u  /* force the tile variant (H, G per tile; any m)                   */
-#define MS_VARIANT_RANGED 4u  /* force the ranged variant (m <= 32, else MS_ERR_UNSUPPORTED)      */
+/* plan flags.  Without a MS_VARIANT_* flag every run picks its variant from
+ * (m, n, key-only / key-value) by the measured rule of DESIGN.md §7; a
+ * MS_VARIANT_* flag makes every run use that one (at most one may be set):
+ *   MS_VARIANT_3K      tile variant  K1 -> K2 -> K3     (3 launches, any m)
+ *   MS_VARIANT_RANGED  CTA ranges    K1r -> K3          (2 launches, m <= 32)
+ *   MS_VARIANT_ONE     cooperative   one kernel         (1 launch,  m <= 32; a
+ *                      grid that cannot be co-resident fails with MS_ERR_CUDA
+ *                      instead of falling back to the ranged variant)
+ * MS_ABLATION_DIRECT: the paper's "Direct" post-scan (Table 4):
+ * no local reorder, every key stored straight to its global position (tile
+ * variant; implemented for MS_DELTA with m <= 32 and m * delta = 2^32 only,
+ * else MS_ERR_UNSUPPORTED) -- a design-space ablation, same result. */
+#define MS_VALIDATE        1u  /* flag precomputed ids >= m on the device; ms_plan_check reports it */
+#define MS_VARIANT_3K      2u
+#define MS_VARIANT_RANGED  4u
+#define MS_VARIANT_ONE     8u
+#define MS_ABLATION_DIRECT 16u
 
-/* Create a plan for up to max_n elements (max_n < 2^32).  with_values != 0
- * plans key-value runs.  Host-only: validates the spec (m range, power-of-two
- * m for MS_LOWBITS, delta >= 1, sorted splitters, id_bytes) and precomputes
- * the bucket-function constants.  Returns MS_ERR_INVALID_ARG on a bad spec. */
+/* Create a plan for up to max_n elements (max_n < 2^32) on CUDA device
+ * `device` (-1: the calling thread's current device; every later call of the
+ * plan switches to that device for its duration).  with_values != 0 plans
+ * key-value runs.  Host-only: validates the spec (m range, power-of-two m for
+ * MS_LOWBITS, delta >= 1, sorted splitters, id_bytes) and the flags, and
+ * precomputes the bucket-function constants.  Returns MS_ERR_INVALID_ARG on a
+ * bad spec or flag combination, MS_ERR_UNSUPPORTED for a variant the spec
+ * cannot use (m > 32 with MS_VARIANT_RANGED / MS_VARIANT_ONE). */
 ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n,
-                         int with_values, uint32_t flags);
+                         int with_values, uint32_t flags, int device);
 
 /* Device workspace bytes ms_run needs for n elements (n <= max_n). */
 ms_status ms_plan_workspace_size(ms_plan_t plan, uint64_t n, size_t *bytes);
 
 /* Tile geometry the plan uses for n elements: tile = T (keys per subproblem),
- * num_tiles = L = ceil(n / T), variant = 0 (tile) or 1 (ranged). */
+ * num_tiles = L = ceil(n / T), variant = 0 (tile, 3 launches), 1 (ranged, 2)
+ * or 2 (ONE, 1) -- the variant a run of n elements (key-value if the plan has
+ * values) takes. */
 ms_status ms_plan_geometry(ms_plan_t plan, uint64_t n, uint32_t *tile, uint64_t *num_tiles,
                            int32_t *variant);
 
@@ -146,8 +166,10 @@ ms_status ms_bucket_ids(ms_plan_t plan, const uint32_t *keys_in, uint64_t n, uin
                         void *stream);
 
 /* Synchronises `stream`, then reports MS_ERR_BUCKET_RANGE if a run on this
- * workspace since the last check saw an id >= m (plans with MS_VALIDATE),
- * clearing the flag; MS_OK otherwise. */
+ * workspace since the last check saw an id >= m (plans with MS_VALIDATE), or
+ * MS_ERR_INVALID_ARG if an ms_postscan_scatter on it met a run beyond its
+ * target's last window (inconsistent win_start / delta: the overflowing part
+ * was not stored), clearing the flag; MS_OK otherwise. */
 ms_status ms_plan_check(ms_plan_t plan, void *workspace, void *stream);
 
 ms_status ms_plan_destroy(ms_plan_t plan);

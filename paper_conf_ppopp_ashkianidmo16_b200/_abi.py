@@ -19,10 +19,14 @@ MS_ERR_ALIGNMENT = -3
 MS_ERR_ALIAS = -4
 MS_ERR_WORKSPACE = -5
 MS_ERR_CUDA = -6
+MS_ERR_NCCL = -7
 MS_ERR_BUCKET_RANGE = -8
 
 MS_LOWBITS, MS_DELTA, MS_SPLITTERS, MS_IDS = 0, 1, 2, 3
-MS_VALIDATE, MS_VARIANT_3K, MS_VARIANT_RANGED = 1, 2, 4
+MS_VALIDATE, MS_VARIANT_3K, MS_VARIANT_RANGED, MS_VARIANT_ONE, MS_ABLATION_DIRECT = 1, 2, 4, 8, 16
+# ms_plan_geometry's variant codes and the kernel launches one ms_run of each enqueues
+VARIANT_TILE, VARIANT_RANGED, VARIANT_ONE = 0, 1, 2
+LAUNCHES = {VARIANT_TILE: 3, VARIANT_RANGED: 2, VARIANT_ONE: 1}
 
 # every symbol include/ms.h declares (tests check the library exports them all)
 EXPORTS = [
@@ -76,7 +80,8 @@ def lib():
                           "there is no CPU fallback for the multisplit")
     L = ctypes.CDLL(LIB_PATH)
     P, U32, U64, I32, SZ = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int32, ctypes.c_size_t
-    L.ms_plan_create.argtypes = [ctypes.POINTER(P), ctypes.POINTER(ms_bucket_spec), U64, ctypes.c_int, U32]
+    L.ms_plan_create.argtypes = [ctypes.POINTER(P), ctypes.POINTER(ms_bucket_spec), U64, ctypes.c_int, U32,
+                                 ctypes.c_int]
     L.ms_plan_workspace_size.argtypes = [P, U64, ctypes.POINTER(SZ)]
     L.ms_plan_workspace_size_host.argtypes = [P, U64, ctypes.POINTER(SZ)]
     L.ms_plan_geometry.argtypes = [P, U64, ctypes.POINTER(U32), ctypes.POINTER(U64), ctypes.POINTER(I32)]

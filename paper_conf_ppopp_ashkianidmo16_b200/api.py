@@ -79,24 +79,29 @@ def _check_tensor(t, name):
         raise ValueError(f"{name} must be contiguous")
 
 
+VARIANT_FLAGS = {None: 0, "3k": _abi.MS_VARIANT_3K, "tile": _abi.MS_VARIANT_3K, "ranged": _abi.MS_VARIANT_RANGED,
+                 "one": _abi.MS_VARIANT_ONE, "direct": _abi.MS_ABLATION_DIRECT}
+
+
 class Plan:
-    """ms_plan_t with a cached device workspace."""
+    """ms_plan_t with a cached device workspace.
+
+    variant: None (chosen per run), "3k"/"tile", "ranged", "one" (MS_VARIANT_*), or
+    "direct" (MS_ABLATION_DIRECT).  device: CUDA ordinal (None = the current device)."""
 
     def __init__(self, spec: BucketSpec, max_n: int, with_values: bool = False, validate: bool = False,
-                 variant: str | None = None):
+                 variant: str | None = None, device: int | None = None):
         L = _abi.lib()
-        flags = _abi.MS_VALIDATE if validate else 0
-        if variant == "3k":
-            flags |= _abi.MS_VARIANT_3K
-        elif variant == "ranged":
-            flags |= _abi.MS_VARIANT_RANGED
+        if variant not in VARIANT_FLAGS:
+            raise ValueError(f"unknown variant {variant!r}")
+        flags = (_abi.MS_VALIDATE if validate else 0) | VARIANT_FLAGS[variant]
         self.spec = spec
         self.max_n = int(max_n)
         self.with_values = bool(with_values)
         self._h = ctypes.c_void_p()
         c = spec._c()
-        check(L.ms_plan_create(ctypes.byref(self._h), ctypes.byref(c), self.max_n, int(with_values), flags),
-              "ms_plan_create")
+        check(L.ms_plan_create(ctypes.byref(self._h), ctypes.byref(c), self.max_n, int(with_values), flags,
+                               -1 if device is None else int(device)), "ms_plan_create")
         self._ws = None
 
     def __del__(self):

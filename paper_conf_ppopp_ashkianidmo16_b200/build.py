@@ -14,8 +14,9 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 OBJ = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libms.so")
-SOURCES = ["ms_api.cu", "ms_dist.cu", "k3p_lowbits.cu", "k3p_shiftc.cu", "k3p_shift.cu", "k3p_delta.cu", "k3p_splitters.cu", "k3p_ids.cu"]
-HEADERS = ["ms_k3_v2.cuh", "ms_kernels.cuh", "ms_device.cuh", "ms_k3_blocked.cuh", "ms_k3_warp.cuh", "ms_k3p_args.h", "ms_ranged.cuh", "ms_k3_lsd.cuh"]
+SOURCES = ["ms_api.cu", "ms_dist.cu", "k3_lowbits.cu", "k3_shiftc.cu", "k3_shift.cu", "k3_delta.cu", "k3_splitters.cu",
+           "k3_ids.cu"]
+HEADERS = ["ms_k3_v2.cuh", "ms_kernels.cuh", "ms_device.cuh", "ms_k3_warp.cuh", "ms_k3p_args.h", "ms_ranged.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr"]

@@ -20,6 +20,9 @@
 
 using namespace ms;
 
+// Variants (include/ms.h): which kernels one ms_run enqueues.
+enum Variant : int { V_TILE = 0, V_RANGED = 1, V_ONE = 2 };
+
 struct ms_plan_s {
   ms_bucket_spec spec;
   uint64_t max_n;
@@ -27,20 +30,13 @@ struct ms_plan_s {
   uint32_t flags;
   BucketParams bp;
   int kkind;  // kernel-level Kind (ms_device.cuh)
-  uint32_t kpt = 16;  // K3 (m <= 32): keys per thread
-  uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt (MS_K3_NT)
-  int ranged = 0;  // CTA-range variant (ms_ranged.cuh, m <= 32): 0 never, 1 when L is large, 2 always
-  int pdl = 1;     // programmatic dependent launch of K2, K3 (MS_PDL=0 disables)
-  // 32 < m <= 256, kinds other than MS_IDS: MS_K3H=1 selects the two-digit K3
-  // (ms_k3_lsd.cuh); measured slower than the warp-ballot K3, so off
-  int k3h = 0;
-  int tile_forced = 0;  // MS_VARIANT_3K flag or MS_VARIANT=tile
-  uint32_t k1s_per_sm = 8;  // splitter K1: persistent CTAs per SM (each builds the bin table once; MS_K1S_PER_SM)
-  int direct = 0;       // ablation MS_K3_DIRECT=1: K3 stores keys straight to global, no local reorder
-  int one_kv = 1;    // ONE for key-value runs: 0 never, 1 when L <= 64 tiles per SM, 2 always (MS_ONE_KV)
-  int one = 1;       // ONE cooperative launch (K3 v2 phase 1 + grid barrier + reverse walk); MS_ONE=0 disables
-  int fuse_k2r = 1;  // ranged variant: range scan folded into K3 (MS_RANGED_K2=1: separate K2r launch)
-  int k3v = 1;     // m <= 32, kinds other than MS_IDS: K3 v2 (ms_k3_v2.cuh); MS_K3V=0 selects the first K3
+  int device;  // CUDA ordinal every call of this plan runs on
+  int sms;     // its SM count
+  uint32_t kpt = 16;    // K3 (m <= 32): keys per thread
+  uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt = 4096
+  int forced = -1;      // MS_VARIANT_* flag: the variant every run uses (-1: chosen per run)
+  int direct = 0;       // MS_ABLATION_DIRECT: K3 stores keys straight to global, no local reorder
+  uint32_t k1s_per_sm = 8;  // splitter K1: persistent CTAs per SM (each builds the bin table once)
   int32_t last_launches;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
   int tracing = 0;     // 0 off, 1 per-stage events, 2 whole-run events only
@@ -83,9 +79,8 @@ uint64_t delta_magic(uint32_t d) { return ~0ull / d + 1; }
 // Rounds per warp R (tile T = 256 R): 16 for m <= 32, 32 above (runs of T/m
 // keys stay >= 32 keys = 128 B); halved while the grid would not fill two
 // waves of 148 SMs (small n is launch/latency bound, not HBM bound).
-int rounds_for(uint32_t m, uint64_t n, uint32_t kpt, bool k3h) {
+int rounds_for(uint32_t m, uint64_t n, uint32_t kpt) {
   if (m <= 32) return (int)kpt;  // blocked-rank K3: T = 256 * kpt for every n
-  if (k3h) return 16;            // persistent two-digit K3 (ms_k3_lsd.cuh): T = 4096 for every n
   int R = 16;
   while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
   return R;
@@ -98,12 +93,12 @@ struct Geometry {
   uint64_t hg_words;   // m * L
   uint64_t chunks;     // K2 CTAs
   size_t off_hg, off_status, off_flag, bytes;
-  size_t off_hc, off_gb;  // CTA-range variant: HC[C][m], GB[C][m] (C <= kMaxRanges), over the H/G region
+  size_t off_hc;          // CTA-range / ONE variants: range counts HC[R][m], over the H/G region
 };
 
 Geometry geometry(const ms_plan_s *p, uint64_t n) {
   Geometry g{};
-  g.R = rounds_for(p->spec.m, n, p->kpt * p->k3nt / 256, p->k3h && p->kkind != IDS);
+  g.R = rounds_for(p->spec.m, n, p->kpt * p->k3nt / 256);
   g.T = 256u * g.R;
   g.L = (n + g.T - 1) / g.T;
   g.hg_words = (uint64_t)p->spec.m * g.L;
@@ -113,12 +108,9 @@ Geometry geometry(const ms_plan_s *p, uint64_t n) {
   g.off_hg = kAlign;
   g.off_status = g.off_hg + align_up(g.hg_words * 4);
   g.bytes = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);
-  if (p->spec.m <= 32) {  // the range arrays reuse the tile arrays' space (never live together)
-    const size_t hw = align_up((size_t)kMaxRangeRows * p->spec.m * 4);
-    const size_t rw = align_up(std::min<uint64_t>(std::max<uint64_t>(g.L, 1), kMaxRanges) * p->spec.m * 4);
+  if (p->spec.m <= 32) {  // the range counts reuse the tile arrays' space (never live together)
     g.off_hc = g.off_hg;
-    g.off_gb = g.off_hc + hw;
-    g.bytes = std::max(g.bytes, g.off_gb + rw);
+    g.bytes = std::max(g.bytes, g.off_hc + align_up((size_t)kMaxRangeRows * p->spec.m * 4));
   }
   return g;
 }
@@ -136,16 +128,18 @@ void set_smem(K kernel, size_t bytes) {
   if (bytes > 48 * 1024) cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
 }
 
-int sm_count() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
+// Every call of a plan runs on the plan's device: switch to it for the call's
+// duration when the calling thread is on another one.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    int cur = -1;
+    if (cudaGetDevice(&cur) == cudaSuccess && cur != dev && cudaSetDevice(dev) == cudaSuccess) prev = cur;
   }
-  return sms;
-}
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
 
 size_t k1_smem(uint32_t m, int kind) {
   return kMaxM * 4 + (kind == SPLITTERS ? kSplBins * 4 : 0) + (size_t)m * kThreads;
@@ -167,7 +161,7 @@ cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *key
                                  : k1_prescan<KIND, KPT, SUBT>;                                     \
     set_smem(k, smem);                                                                             \
     uint64_t grid = (g.L + SUBT - 1) / SUBT;                                                       \
-    if (KIND == SPLITTERS && p->spec.m <= 32) grid = std::min<uint64_t>(grid, (uint64_t)p->k1s_per_sm * sm_count()); \
+    if (KIND == SPLITTERS && p->spec.m <= 32) grid = std::min<uint64_t>(grid, (uint64_t)p->k1s_per_sm * p->sms); \
     k<<<(unsigned)grid, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, zero_words, \
                                              flag);                                                \
   }
@@ -196,41 +190,24 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
 
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
-                        uint32_t *vo, uint32_t n, cudaStream_t s, int ranged = 0,
+                        uint32_t *vo, uint32_t n, uint32_t *flag, cudaStream_t s, int ranged = 0,
                         uint32_t *grid_out = nullptr, int pdl = 0, const RangeScan *rs = nullptr) {
   K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
-            p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, sm_count(), s};
+            p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, p->sms, s};
   a.ranged = ranged;
   a.grid_out = grid_out;
   a.pdl = pdl;
   a.direct = p->direct;
+  a.flag = flag;
   if (rs) a.rs = *rs;
-  if (p->spec.m <= 32 && p->k3v && p->kkind != IDS) {  // K3 v2 (ms_k3_v2.cuh)
+  if (p->spec.m <= 32) {  // K3 v2 (ms_k3_v2.cuh), one TU per kind
     switch (p->kkind) {
       case LOWBITS: return k3v_launch_lowbits(a);
       case SHIFTC: return k3v_launch_shiftc(a);
       case SHIFT: return k3v_launch_shift(a);
       case DELTA: return k3v_launch_delta(a);
-      default: return k3v_launch_splitters(a);
-    }
-  }
-  if (p->spec.m <= 32) {  // persistent blocked-rank K3 (ms_k3_blocked.cuh), one TU per kind
-    switch (p->kkind) {
-      case LOWBITS: return k3p_launch_lowbits(a);
-      case SHIFTC: return k3p_launch_shiftc(a);
-      case SHIFT: return k3p_launch_shift(a);
-      case DELTA: return k3p_launch_delta(a);
-      case SPLITTERS: return k3p_launch_splitters(a);
-      default: return k3p_launch_ids(a);
-    }
-  }
-  if (p->k3h && p->kkind != IDS) {  // 32 < m <= 256: two-digit local multisplit (ms_k3_lsd.cuh)
-    switch (p->kkind) {
-      case LOWBITS: return k3h_launch_lowbits(a);
-      case SHIFTC: return k3h_launch_shiftc(a);
-      case SHIFT: return k3h_launch_shift(a);
-      case DELTA: return k3h_launch_delta(a);
-      default: return k3h_launch_splitters(a);
+      case SPLITTERS: return k3v_launch_splitters(a);
+      default: return k3v_launch_ids(a);
     }
   }
   switch (p->kkind) {  // m > 32: warp-ballot K3 (ms_k3_warp.cuh)
@@ -244,14 +221,14 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
 }
 
 // K1r: k sub-ranges per range so that the grid has ~8 CTAs of 256 threads per SM
-uint32_t k1r_split(uint32_t C) {
-  return std::max<uint32_t>(1u, std::min<uint32_t>(8u * (uint32_t)sm_count() / C, kMaxRangeRows / C));
+uint32_t k1r_split(const ms_plan_s *p, uint32_t C) {
+  return std::max<uint32_t>(1u, std::min<uint32_t>(8u * (uint32_t)p->sms / C, kMaxRangeRows / C));
 }
 
 template <int KIND>
 cudaError_t launch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, const uint32_t *keys, const void *ids,
                        uint32_t n, uint32_t *HC, uint32_t *flag, cudaStream_t s) {
-  const uint32_t k = k1r_split(C);
+  const uint32_t k = k1r_split(p, C);
   auto kern = k1r_prescan<KIND, 256>;
   const size_t smem = k1r_smem(p->spec.m, KIND, 256);
   set_smem(kern, smem);
@@ -271,8 +248,18 @@ cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, cons
   }
 }
 
-bool use_ranged(const ms_plan_s *p, uint64_t L) {
-  return p->ranged == 2 || (p->ranged == 1 && L >= 8ull * (uint64_t)sm_count());
+// The variant a run of L tiles uses (measured on B200).  m > 32 and the Direct
+// ablation: tile.  Forced by a MS_VARIANT_* plan flag: that one.  Otherwise ONE for every
+// key-only run and for key-value runs of up to 64 tiles per SM (C3, n = 2^25: 192 -> 207
+// G keys/s); above that the CTA-range variant for m <= 16 (mean bucket run per tile >= 256
+// keys; NSkv-like m4..16 KV 321 vs 305 with ONE), the tile variant for 16 < m <= 32 (shorter
+// runs: concurrently processed tiles write ADJACENT runs of every bucket).
+int choose_variant(const ms_plan_s *p, uint64_t L, bool kv) {
+  if (p->spec.m > 32 || p->direct) return V_TILE;
+  if (p->forced >= 0) return p->forced;
+  if (!kv || L <= 64ull * (uint64_t)p->sms) return V_ONE;
+  if (p->k3nt * p->kpt >= 256u * p->spec.m && L >= 8ull * (uint64_t)p->sms) return V_RANGED;
+  return V_TILE;
 }
 
 ms_status check_ws(const ms_plan_s *p, uint64_t n, void *ws, size_t ws_bytes, Geometry *g) {
@@ -305,21 +292,25 @@ const char *ms_status_string(ms_status s) {
     case MS_ERR_ALIAS: return "output overlaps input";
     case MS_ERR_WORKSPACE: return "workspace missing or too small";
     case MS_ERR_CUDA: return "CUDA error";
+    case MS_ERR_NCCL: return "NCCL error";
     case MS_ERR_BUCKET_RANGE: return "bucket id >= m";
     default: return "unknown status";
   }
 }
 
 ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n,
-                         int with_values, uint32_t flags) {
+                         int with_values, uint32_t flags, int device) {
   if (!plan || !spec) return MS_ERR_INVALID_ARG;
   *plan = nullptr;
   const uint32_t m = spec->m;
   if (m < 1 || m > (uint32_t)kMaxM) return MS_ERR_INVALID_ARG;
   if (max_n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
-  if ((flags & MS_VARIANT_3K) && (flags & MS_VARIANT_RANGED)) return MS_ERR_INVALID_ARG;
-  if (flags & ~(MS_VALIDATE | MS_VARIANT_3K | MS_VARIANT_RANGED)) return MS_ERR_INVALID_ARG;
-  if ((flags & MS_VARIANT_RANGED) && m > 32) return MS_ERR_UNSUPPORTED;
+  constexpr uint32_t kVariants = MS_VARIANT_3K | MS_VARIANT_RANGED | MS_VARIANT_ONE;
+  if (flags & ~(MS_VALIDATE | kVariants | MS_ABLATION_DIRECT)) return MS_ERR_INVALID_ARG;
+  const uint32_t vf = flags & kVariants;
+  if (vf & (vf - 1)) return MS_ERR_INVALID_ARG;  // at most one variant flag
+  if ((flags & MS_ABLATION_DIRECT) && vf) return MS_ERR_INVALID_ARG;
+  if ((flags & (MS_VARIANT_RANGED | MS_VARIANT_ONE)) && m > 32) return MS_ERR_UNSUPPORTED;
   BucketParams bp;
   memset(&bp, 0, sizeof(bp));
   int kkind = spec->kind;
@@ -361,6 +352,18 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
       break;
     default: return MS_ERR_INVALID_ARG;
   }
+  // the Direct ablation is instantiated for one bucket kind only (DELTA with m * delta = 2^32)
+  if ((flags & MS_ABLATION_DIRECT) && (m > 32 || kkind != SHIFT)) return MS_ERR_UNSUPPORTED;
+  if (device < -1) return MS_ERR_INVALID_ARG;
+  if (device == -1 && cudaGetDevice(&device) != cudaSuccess) {
+    cudaGetLastError();
+    device = 0;  // no usable device yet (host-only use of the plan): ordinal 0
+  }
+  int sms = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || sms <= 0) {
+    cudaGetLastError();
+    sms = 148;  // B200
+  }
   ms_plan_s *p = new (std::nothrow) ms_plan_s;
   if (!p) return MS_ERR_INVALID_ARG;
   p->spec = *spec;
@@ -370,50 +373,12 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->flags = flags;
   p->bp = bp;
   p->kkind = kkind;
+  p->device = device;
+  p->sms = sms;
   p->last_launches = 0;
-  // K3 CTA size (m <= 32), measured per workload: 256 threads
-  // (T = 4096) for m > 16 with one-instruction ids, 128 (T = 2048) otherwise
-  p->k3nt = (m > 16 && (kkind == SHIFT || kkind == SHIFTC || kkind == LOWBITS)) ? 256u : 128u;
-  if (kkind != IDS) p->k3nt = 256u;  // K3 v2: 256 threads (T = 4096) measured best for every m <= 32
-  // ablation overrides: MS_DEBUG_K3=1 drops K3's global stores;
-  // MS_K3_REVERSE=1 walks K3's tiles last-to-first
-  if (const char *e = getenv("MS_DEBUG_K3")) p->bp.dbg = (uint32_t)atoi(e);
-  if (const char *e = getenv("MS_K3_REVERSE")) p->bp.reverse = atoi(e) ? 1u : 0u;
-  if (const char *e = getenv("MS_K3_NT")) p->k3nt = atoi(e) == 128 ? 128u : 256u;
-  // K3 v2 at 128 threads runs 32 keys per thread (same T = 4096)
-  if (kkind != IDS && p->k3nt == 128) p->kpt = 32;
-  // variant: CTA ranges for m <= 32 when a tile's mean bucket
-  // run is >= 256 keys (1 KB).  With shorter runs the strided tile walk wins:
-  // its concurrently processed tiles write ADJACENT runs of every bucket (m
-  // dense write streams), while contiguous ranges scatter them over C*m
-  // streams.  Forced either way by MS_VARIANT_3K / MS_VARIANT_RANGED (and
-  // MS_VARIANT=tile|ranged in the environment, for A/B measurements).
-  // Small inputs (L < 8 tiles per SM) keep the tile variant: a range is then
-  // only one or two tiles and the per-range setup is pure overhead.
-  p->ranged = (m <= 32 && p->k3nt * p->kpt >= 256u * m) ? 1 : 0;
-  if (const char *e = getenv("MS_VARIANT")) {
-    if (strcmp(e, "tile") == 0) p->ranged = 0;
-    if (strcmp(e, "ranged") == 0 && m <= 32) p->ranged = 2;
-  }
-  if (flags & MS_VARIANT_3K) p->ranged = 0;
-  p->tile_forced = (flags & MS_VARIANT_3K) ? 1 : 0;
-  if (const char *e = getenv("MS_VARIANT"))
-    if (strcmp(e, "tile") == 0) p->tile_forced = 1;
-  if (const char *e = getenv("MS_K1S_PER_SM")) p->k1s_per_sm = std::max(1, std::min(16, atoi(e)));
-  if (const char *e = getenv("MS_K3_DIRECT")) {
-    p->direct = atoi(e) ? 1 : 0;
-    if (p->direct) {
-      p->tile_forced = 1;  // the ablation runs the 3-kernel tile variant
-      p->ranged = 0;
-    }
-  }
-  if (flags & MS_VARIANT_RANGED) p->ranged = 2;
-  if (const char *e = getenv("MS_PDL")) p->pdl = atoi(e) ? 1 : 0;
-  if (const char *e = getenv("MS_K3V")) p->k3v = atoi(e) ? 1 : 0;
-  if (const char *e = getenv("MS_ONE")) p->one = atoi(e) ? 1 : 0;
-  if (const char *e = getenv("MS_ONE_KV")) p->one_kv = std::max(0, std::min(2, atoi(e)));
-  if (const char *e = getenv("MS_K3H")) p->k3h = atoi(e) ? 1 : 0;
-  if (const char *e = getenv("MS_RANGED_K2")) p->fuse_k2r = atoi(e) ? 0 : 1;
+  p->forced = (flags & MS_VARIANT_3K) ? V_TILE : (flags & MS_VARIANT_RANGED) ? V_RANGED
+            : (flags & MS_VARIANT_ONE) ? V_ONE : -1;
+  p->direct = (flags & MS_ABLATION_DIRECT) ? 1 : 0;
   *plan = p;
   return MS_OK;
 }
@@ -437,7 +402,7 @@ ms_status ms_plan_geometry(ms_plan_t p, uint64_t n, uint32_t *tile, uint64_t *nu
   Geometry g = geometry(p, n);
   if (tile) *tile = g.T;
   if (num_tiles) *num_tiles = g.L;
-  if (variant) *variant = use_ranged(p, g.L) ? 1 : 0;
+  if (variant) *variant = choose_variant(p, g.L, p->kv != 0);
   return MS_OK;
 }
 
@@ -478,6 +443,7 @@ ms_status ms_prescan(ms_plan_t p, const uint32_t *keys_in, const void *ids, uint
   Geometry g;
   if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
   if (n == 0) return MS_OK;
+  DeviceGuard dg(p->device);
   char *w = (char *)ws;
   cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, H, nullptr, 0,
                               (uint32_t *)(w + g.off_flag), (cudaStream_t)stream);
@@ -491,12 +457,13 @@ ms_status ms_scan(ms_plan_t p, uint32_t *HG, uint64_t n, uint32_t *offsets, void
   Geometry g;
   ms_status st = check_ws(p, n, ws, ws_bytes, &g);
   if (st != MS_OK) return st;
+  if (n > 0 && !HG) return MS_ERR_INVALID_ARG;
+  DeviceGuard dg(p->device);
   cudaStream_t s = (cudaStream_t)stream;
   if (n == 0) {
     if (offsets && cudaMemsetAsync(offsets, 0, (p->spec.m + 1) * 4, s) != cudaSuccess) return MS_ERR_CUDA;
     return MS_OK;
   }
-  if (!HG) return MS_ERR_INVALID_ARG;
   char *w = (char *)ws;
   uint64_t *status = (uint64_t *)(w + g.off_status);
   if (cudaMemsetAsync(status, 0, g.chunks * 8, s) != cudaSuccess) return MS_ERR_CUDA;
@@ -518,15 +485,16 @@ ms_status ms_postscan(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals
   Geometry g;
   if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
   if (n == 0) return MS_OK;
+  DeviceGuard dg(p->device);
   cudaError_t e = dispatch_k3(p, g, keys_in, vals_in, ids, G, keys_out, vals_out, (uint32_t)n,
-                              (cudaStream_t)stream);
+                              (uint32_t *)((char *)ws + g.off_flag), (cudaStream_t)stream);
   return e == cudaSuccess ? MS_OK : MS_ERR_CUDA;
 }
 
 ms_status ms_postscan_scatter(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, const uint32_t *G,
                               uint64_t n, const ms_scatter_target *t, void *ws, size_t ws_bytes, void *stream) {
   if (!p) return MS_ERR_INVALID_ARG;
-  if (p->spec.m > 32 || p->kkind == IDS || !p->k3v) return MS_ERR_UNSUPPORTED;
+  if (p->spec.m > 32 || p->kkind == IDS || p->direct) return MS_ERR_UNSUPPORTED;
   ms_status st = check_common(p, keys_in, nullptr, n);
   if (st != MS_OK) return st;
   if (!t || t->nranks < 1 || t->nranks > MS_MAX_PEERS) return MS_ERR_INVALID_ARG;
@@ -542,6 +510,7 @@ ms_status ms_postscan_scatter(ms_plan_t p, const uint32_t *keys_in, const uint32
   if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
   if (n == 0) return MS_OK;
   if (!G) return MS_ERR_INVALID_ARG;
+  DeviceGuard dg(p->device);
   DistTarget d{};
   d.P = t->nranks;
   for (int32_t r = 0; r < t->nranks; ++r) {
@@ -551,8 +520,9 @@ ms_status ms_postscan_scatter(ms_plan_t p, const uint32_t *keys_in, const uint32
   for (int32_t r = 0; r <= t->nranks; ++r) d.wst[r] = t->win_start[r];
   for (uint32_t b = 0; b < p->spec.m; ++b) d.delta[b] = t->delta[b];
   K3pArgs a{keys_in, vals_in, nullptr, G, nullptr, nullptr, (uint32_t)n, (uint32_t)g.L, p->spec.m,
-            p->spec.id_bytes, p->kpt, p->k3nt, &p->bp, sm_count(), (cudaStream_t)stream};
+            p->spec.id_bytes, p->kpt, p->k3nt, &p->bp, p->sms, (cudaStream_t)stream};
   a.ds = &d;
+  a.flag = (uint32_t *)((char *)ws + g.off_flag);  // a run past win_start[P] sets bit 1 (ms_plan_check)
   cudaError_t e;
   switch (p->kkind) {
     case LOWBITS: e = k3v_launch_lowbits(a); break;
@@ -582,6 +552,7 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
     return MS_ERR_ALIAS;
   Geometry g;
   if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
+  DeviceGuard dg(p->device);
   cudaStream_t s = (cudaStream_t)stream;
   p->last_launches = 0;
   if (n == 0) {
@@ -592,72 +563,54 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   uint32_t *HG = (uint32_t *)(w + g.off_hg);
   uint64_t *status = (uint64_t *)(w + g.off_status);
   uint32_t *flag = (uint32_t *)(w + g.off_flag);
+  uint32_t *HC = (uint32_t *)(w + g.off_hc);
   if ((p->flags & MS_VALIDATE) && p->spec.kind == MS_IDS &&
       cudaMemsetAsync(flag, 0, 4, s) != cudaSuccess)
     return MS_ERR_CUDA;
   cudaEvent_t *ev = trace_next(p);
   if (ev) cudaEventRecord(ev[0], s);
   // K2 and K3 use programmatic dependent launch unless per-stage events sit
-  // between the kernels (tracing == 1) or MS_PDL=0
-  const bool pdl = p->pdl && p->tracing != 1;
-  // ONE cooperative launch (K3 v2 ONE mode), measured: key-only runs of the ranged
-  // variant, and key-only runs too small for it (L < 8 tiles per SM: 3 launches -> 1)
-  // (m <= 32 key-only: ONE beats the 3-kernel tile variant too -- NSko 410 -> 422 G keys/s -- unless
-  // the tile variant is forced by MS_VARIANT_3K / MS_VARIANT=tile)
-  // key-value: ONE at up to 64 tiles per SM (C3, n = 2^25: 192 -> 207 G keys/s), not above
-  // (NSkv, n = 2^28: 293 -> 276 -- the two/three-launch paths stream better there)
-  const bool one = p->one && p->k3v && p->kkind != IDS && p->spec.m <= 32 && !p->tile_forced &&
-                   (!vals_in || p->one_kv == 2 || (p->one_kv == 1 && g.L <= 64ull * (uint64_t)sm_count()));
-  if (one) {
-    uint32_t *HC = (uint32_t *)(w + g.off_hc);
+  // between the kernels (tracing == 1)
+  const bool pdl = p->tracing != 1;
+  int variant = choose_variant(p, g.L, vals_in != nullptr);
+  if (variant == V_ONE) {  // ONE cooperative launch: counts, grid barrier, range scan, post-scan
     const RangeScan rs{HC, offsets, 0, 1};
     if (ev && p->tracing == 1) {
       cudaEventRecord(ev[1], s);
       cudaEventRecord(ev[2], s);
     }
-    const cudaError_t e1 = dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 2,
-                                       nullptr, 0, &rs);
+    const cudaError_t e1 = dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, flag,
+                                       s, 2, nullptr, 0, &rs);
     if (e1 == cudaSuccess) {
       if (ev) cudaEventRecord(ev[3], s);
       p->last_launches = 1;
       return MS_OK;
     }
-    // the grid could not be made co-resident (e.g. the GPU is partitioned / shared): clear the
-    // launch error and take the multi-launch path below (same result)
-    if (e1 != cudaErrorCooperativeLaunchTooLarge) return MS_ERR_CUDA;
+    // the grid could not be made co-resident (e.g. the GPU is partitioned / shared): unless ONE
+    // was forced, clear the launch error and take the two-launch ranged variant (same result)
+    if (e1 != cudaErrorCooperativeLaunchTooLarge || p->forced == V_ONE) return MS_ERR_CUDA;
     cudaGetLastError();
+    variant = V_RANGED;
   }
-  if (use_ranged(p, g.L)) {  // K1r -> K2r -> K3 over C contiguous tile ranges (ms_ranged.cuh)
+  if (variant == V_RANGED) {  // K1r -> K3 over C contiguous tile ranges (ms_ranged.cuh); the range
+                              // scan runs in K3's prologue
     uint32_t C = 0;
-    if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 1, &C) != cudaSuccess ||
+    if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, flag, s, 1, &C) !=
+            cudaSuccess ||
         C == 0)
       return MS_ERR_CUDA;
-    uint32_t *HC = (uint32_t *)(w + g.off_hc), *GB = (uint32_t *)(w + g.off_gb);
     if (dispatch_k1r(p, g, C, keys_in, ids, (uint32_t)n, HC, flag, s) != cudaSuccess) return MS_ERR_CUDA;
-    if (ev && p->tracing == 1) cudaEventRecord(ev[1], s);
-    const uint32_t ksub = k1r_split(C), R = C * ksub;
-    if (p->fuse_k2r) {  // K1r -> K3 (the range scan runs in K3's prologue): two launches
-      if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
-      const RangeScan rs{HC, offsets, R, ksub};
-      if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, s, 1, nullptr, pdl,
-                      &rs) != cudaSuccess)
-        return MS_ERR_CUDA;
-      if (ev) cudaEventRecord(ev[3], s);
-      p->last_launches = 2;
-      return MS_OK;
+    if (ev && p->tracing == 1) {
+      cudaEventRecord(ev[1], s);
+      cudaEventRecord(ev[2], s);
     }
-    const size_t smem2 = (size_t)R * p->spec.m * 4;
-    set_smem(k2r_scan, smem2);
-    if (launch_ex(pdl, k2r_scan, dim3(1), dim3(kR2Threads), smem2, s, (const uint32_t *)HC, GB, R, ksub, p->spec.m,
-                  std::max<uint32_t>(1, ceil_log2(p->spec.m)), offsets, (uint32_t)n) != cudaSuccess ||
-        cudaGetLastError() != cudaSuccess)
-      return MS_ERR_CUDA;
-    if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
-    if (dispatch_k3(p, g, keys_in, vals_in, ids, GB, keys_out, vals_out, (uint32_t)n, s, 1, nullptr, pdl) !=
-        cudaSuccess)
+    const uint32_t ksub = k1r_split(p, C);
+    const RangeScan rs{HC, offsets, C * ksub, ksub};
+    if (dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, flag, s, 1, nullptr, pdl,
+                    &rs) != cudaSuccess)
       return MS_ERR_CUDA;
     if (ev) cudaEventRecord(ev[3], s);
-    p->last_launches = 3;
+    p->last_launches = 2;
     return MS_OK;
   }
   cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, status, (uint32_t)g.chunks, flag, s);
@@ -671,7 +624,7 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   // K3 after the many-CTA K2 of the tile variant: PDL only for key-only runs
   // (measured: an early-resident key-value K3 -- 2 CTAs with
   // the whole register file per SM -- costs ~6 % at n = 2^28)
-  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, s, 0, nullptr,
+  e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, flag, s, 0, nullptr,
                   pdl && vals_in == nullptr);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev) cudaEventRecord(ev[3], s);
@@ -701,6 +654,7 @@ ms_status ms_run_host(ms_plan_t p, const uint32_t *keys_h, const uint32_t *vals_
   ms_plan_workspace_size_host(p, n, &need);
   if (!ws || ws_bytes < need) return MS_ERR_WORKSPACE;
   if (misaligned(ws)) return MS_ERR_ALIGNMENT;
+  DeviceGuard dg(p->device);
   cudaStream_t s = (cudaStream_t)stream;
   Geometry g = geometry(p, n);
   char *w = (char *)ws + g.bytes;
@@ -736,6 +690,7 @@ ms_status ms_bucket_ids(ms_plan_t p, const uint32_t *keys_in, uint64_t n, uint32
   if (p->spec.kind == MS_IDS) return MS_ERR_UNSUPPORTED;
   if (misaligned(keys_in) || misaligned(out_ids)) return MS_ERR_ALIGNMENT;
   if (n == 0) return MS_OK;
+  DeviceGuard dg(p->device);
   cudaStream_t s = (cudaStream_t)stream;
   unsigned grid = (unsigned)std::min<uint64_t>((n + kThreads - 1) / kThreads, 148ull * 16);
   switch (p->kkind) {
@@ -750,13 +705,14 @@ ms_status ms_bucket_ids(ms_plan_t p, const uint32_t *keys_in, uint64_t n, uint32
 
 ms_status ms_plan_check(ms_plan_t p, void *ws, void *stream) {
   if (!p || !ws) return MS_ERR_INVALID_ARG;
+  DeviceGuard dg(p->device);
   cudaStream_t s = (cudaStream_t)stream;
   uint32_t host = 0;
   if (cudaMemcpyAsync(&host, ws, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess) return MS_ERR_CUDA;
   if (cudaStreamSynchronize(s) != cudaSuccess) return MS_ERR_CUDA;
   if (host) {
     if (cudaMemsetAsync(ws, 0, 4, s) != cudaSuccess) return MS_ERR_CUDA;
-    return MS_ERR_BUCKET_RANGE;
+    return (host & 2u) ? MS_ERR_INVALID_ARG : MS_ERR_BUCKET_RANGE;
   }
   return MS_OK;
 }

@@ -31,8 +31,6 @@ struct BucketParams {
   uint32_t logm;      // ceil(log2 m): splitter search steps
   uint32_t id_bytes;  // IDS: 1 or 4
   uint32_t validate;  // IDS: flag ids >= m
-  uint32_t dbg;       // ablation switch (MS_DEBUG_K3): 0 normal
-  uint32_t reverse;   // K3 walks tiles last-to-first (L2 reuse of K1's last reads)
   uint32_t spl[kMaxM];
 };
 

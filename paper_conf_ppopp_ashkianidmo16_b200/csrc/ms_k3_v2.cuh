@@ -88,11 +88,16 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *tm, in
 // G counting down from the range's end.
 // DIRECT (ablation, SURVEY NEXT-2 / the paper's "Direct" method of Table 4): no local reorder --
 // every key is stored from registers straight to its global position G_j + local offset.
+// IDS (precomputed ids, IDB = 1 or 4 bytes per id): the ids of a thread's block are read
+// straight from global memory (16 B / 64 B per 16 keys, next to the TMA-staged keys), clamped
+// to m-1 (a contract violation never indexes outside the counters) and flagged in *flag when
+// p.validate; ONE's phase 1 counts from the ids alone (1 or 4 B per key instead of 4).
 template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, int MINB, int KPT, bool ONE = false,
-          bool DIRECT = false>
+          bool DIRECT = false, int IDB = 0>
 __global__ void __launch_bounds__(NT, MINB)
 k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv,
              const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
+             const void *__restrict__ ids, uint32_t *__restrict__ flag,
              const uint32_t *__restrict__ G, uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
              uint32_t n, uint32_t L, const __grid_constant__ BucketParams p,
              const __grid_constant__ RangeScan rs, const __grid_constant__ DistTarget ds) {
@@ -101,7 +106,44 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   constexpr int NW = NT / 32;
   constexpr int NCH = K / 4;  // 16-byte chunks per thread block
   constexpr int LOGNT = NT == 256 ? 8 : 7;
-  constexpr bool KEEP_ID = KIND == SPLITTERS || KIND == DELTA;  // multi-instruction ids are kept, not recomputed
+  // multi-instruction (and precomputed) ids are kept in registers, one byte per key, not recomputed
+  constexpr bool KEEP_ID = KIND == SPLITTERS || KIND == DELTA || KIND == IDS;
+  static_assert(KIND != IDS || IDB == 1 || IDB == 4, "IDS needs IDB = 1 or 4");
+  const uint32_t mm4 = p.mmask * 0x01010101u;  // IDS: per-byte clamp bound
+  uint32_t bad = 0;                            // IDS: some raw id > m - 1 (validation)
+  // IDS: clamp 4 raw u32 ids into one word of 4 byte ids
+  auto clamp_pack = [&](uint32_t a, uint32_t b, uint32_t c, uint32_t d) -> uint32_t {
+    bad |= (a > p.mmask) | (b > p.mmask) | (c > p.mmask) | (d > p.mmask);
+    return min(a, p.mmask) | (min(b, p.mmask) << 8) | (min(c, p.mmask) << 16) | (min(d, p.mmask) << 24);
+  };
+  auto clamp4 = [&](uint32_t w) -> uint32_t {  // 4 raw u8 ids
+    bad |= __vcmpgtu4(w, mm4);
+    return __vminu4(w, mm4);
+  };
+  // IDS: byte ids of the nch4 * 4 keys from key index e (16-byte aligned, all valid) into w[]
+  auto load_ids_full = [&](uint64_t e, uint32_t *w, int nch4) {
+    if constexpr (IDB == 1) {
+      const uint4 x = __ldcs(reinterpret_cast<const uint4 *>(static_cast<const uint8_t *>(ids) + e));
+      const uint32_t xx[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+        if (c < nch4) w[c] = clamp4(xx[c]);
+    } else {
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+        if (c < nch4) {
+          const uint4 x = __ldcs(reinterpret_cast<const uint4 *>(static_cast<const uint32_t *>(ids) + e) + c);
+          w[c] = clamp_pack(x.x, x.y, x.z, x.w);
+        }
+    }
+  };
+  auto load_id1 = [&](uint64_t i) -> uint32_t {  // one id, clamped
+    uint32_t v;
+    if constexpr (IDB == 1) v = static_cast<const uint8_t *>(ids)[i];
+    else v = static_cast<const uint32_t *>(ids)[i];
+    bad |= v > p.mmask;
+    return min(v, p.mmask);
+  };
   extern __shared__ uint8_t smraw[];
   // align to 1024 B by offsetting the shared pointer itself (an integer round
   // trip would turn every access below into a generic LD/ST)
@@ -144,7 +186,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   const uint32_t ptail = ONE ? iters - nf : 0;  // 0 or 1
   // ONE, key-only (two stages): phase 1 reads the keys through the TMA stages too (measured
   // better than plain loads: C2 389 vs 371 G keys/s); key-value (one stage): plain coalesced loads
-  constexpr bool P1TMA = ONE && !KV;
+  constexpr bool P1TMA = ONE && !KV && KIND != IDS;
   // TMA sequence numbers: ONE keys: [P1TMA: phase 1 forward over the nf full tiles, then] phase 2
   // reverse; ONE values: phase 2 only.  Otherwise sequence = iteration.
   auto seq_tile = [&](uint32_t sq, bool values) -> uint64_t {
@@ -223,10 +265,11 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     };
     zero_cnt();
     __syncthreads();
-    auto count1 = [&](uint32_t key) {
-      const uint32_t a = ccol + id_of(key) * RS;
+    auto count_id = [&](uint32_t id) {
+      const uint32_t a = ccol + id * RS;
       sts_u16(a, lds_u16(a) + 1);
     };
+    auto count1 = [&](uint32_t key) { count_id(id_of(key)); };
     // counting needs no key-to-thread order: coalesced 128-bit loads (chunk j*NT + tid of the
     // tile), the next tile's loads issued before this one is counted (register double buffer)
     auto ld = [&](uint32_t sq, uint4 *dst) {
@@ -255,9 +298,27 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
         if ((sq & 2047u) == 2047u) fold();
       }
     }
-    uint4 xa[NCH], xb[NCH];
-    if (!P1TMA && nf) ld(0, xa);
-    for (uint32_t sq = 0; !P1TMA && sq < nf;) {
+    if constexpr (KIND == IDS) {  // precomputed ids: phase 1 reads only the ids (coalesced 16-byte chunks)
+      constexpr int CH = IDB == 1 ? 1 : NCH;  // 16-byte chunks per thread per tile
+      for (uint32_t sq = 0; sq < nf; ++sq) {
+        const uint64_t tb = (r0 + sq) * T;
+#pragma unroll
+        for (int c = 0; c < CH; ++c) {
+          uint32_t w[4];
+          load_ids_full(tb + (uint64_t)(IDB == 1 ? 16 : 4) * (c * NT + tid), w, IDB == 1 ? 4 : 1);
+#pragma unroll
+          for (int q = 0; q < (IDB == 1 ? 4 : 1); ++q) {
+            count_id(w[q] & 255u); count_id((w[q] >> 8) & 255u);
+            count_id((w[q] >> 16) & 255u); count_id(w[q] >> 24);
+          }
+        }
+        if ((sq & 2047u) == 2047u) fold();
+      }
+    }
+    constexpr bool P1LD = !P1TMA && KIND != IDS;  // key-value, computed ids: plain loads of the keys
+    uint4 xa[P1LD ? NCH : 1], xb[P1LD ? NCH : 1];
+    if (P1LD && nf) ld(0, xa);
+    for (uint32_t sq = 0; P1LD && sq < nf;) {
       if (sq + 1 < nf) ld(sq + 1, xb);
       cnt4(xa);
       if ((sq & 2047u) == 2047u) fold();
@@ -271,7 +332,10 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       const uint64_t base = (r0 + nf) * T;
       const uint32_t nt = (uint32_t)(n - base);
       for (uint32_t q = 0; q < (uint32_t)K; ++q)
-        if (b0 + q < nt) count1(__ldg(keys + base + b0 + q));
+        if (b0 + q < nt) {
+          if constexpr (KIND == IDS) count_id(load_id1(base + b0 + q));
+          else count1(__ldg(keys + base + b0 + q));
+        }
     }
     fold();
     if (tid < m) const_cast<uint32_t *>(rs.HC)[(uint64_t)blockIdx.x * m + tid] = tot_s[tid];
@@ -284,12 +348,9 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     if (row < m) grun += tot_s[row];  // the reverse walk counts down from the range's end
     __syncthreads();
   } else if constexpr (RANGED) {
-    if (rs.HC != nullptr) {  // K2r folded in: this range's G from K1r's rows (keys_s is free until tile 0)
-      grun = range_base<NT, LOGMP>(rs, m, blockIdx.x, n, keys_s, row);
-      __syncthreads();
-    } else if (iters && row < m) {
-      grun = __ldg(G + (uint64_t)blockIdx.x * m + row);
-    }
+    // the range scan (Eq. (2) terms 1+2 over ranges) from K1r's rows (keys_s is free until tile 0)
+    grun = range_base<NT, LOGMP>(rs, m, blockIdx.x, n, keys_s, row);
+    __syncthreads();
   } else {
     if (iters && tid < m) gnext = __ldg(G + (uint64_t)tid * L + tile_of(0));
   }
@@ -347,20 +408,35 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     }
     uint32_t rk[NCH];                   // ranks (< K), one byte each
     uint32_t idk[KEEP_ID ? NCH : 1];    // kept ids, one byte each
+    if constexpr (KIND == IDS) {
+      if constexpr (FULL) {
+        load_ids_full(base + b0, idk, 4);
+      } else {
+#pragma unroll
+        for (int c = 0; c < NCH; ++c) {
+          uint32_t t4[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) t4[j] = b0 + 4 * c + j < nt ? load_id1(base + b0 + 4 * c + j) : 0u;
+          idk[c] = t4[0] | (t4[1] << 8) | (t4[2] << 16) | (t4[3] << 24);
+        }
+      }
+    }
 #pragma unroll
     for (int c = 0; c < NCH; ++c) {
       const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
       rk[c] = 0u;
-      if constexpr (KEEP_ID) idk[c] = 0u;
+      if constexpr (KEEP_ID && KIND != IDS) idk[c] = 0u;
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         if (FULL || b0 + 4 * c + j < nt) {
-          const uint32_t id = id_of(kk[j]);
+          uint32_t id;
+          if constexpr (KIND == IDS) id = __byte_perm(idk[c], 0u, 0x4440u + j);
+          else id = id_of(kk[j]);
           const uint32_t a = ccol + id * RS;
           const uint32_t r = lds_u16(a);
           sts_u16(a, r + 1);
           rk[c] |= r << (8 * j);
-          if constexpr (KEEP_ID) idk[c] |= id << (8 * j);
+          if constexpr (KEEP_ID && KIND != IDS) idk[c] |= id << (8 * j);
         }
       }
     }
@@ -541,6 +617,10 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
         uint32_t src = Pj[b];
         uint64_t gs = (uint64_t)Gj[b] + ds.delta[b];
         while (left) {
+          if (gs >= ds.wst[ds.P]) {  // inconsistent target (a run past the last window): store nothing
+            atomicOr(flag, 2u);      // more, report it through ms_plan_check
+            break;
+          }
           uint32_t r = 0;
           for (int i = 1; i < ds.P; ++i) r += gs >= ds.wst[i] ? 1u : 0u;
           const uint64_t room = ds.wst[r + 1] - gs;
@@ -617,6 +697,9 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     for (uint32_t it = 0; it < iters_full; ++it) tile_body(it, std::true_type{});
     if (has_tail) tile_body(iters_full, std::false_type{});
   }
+  if constexpr (KIND == IDS) {
+    if (p.validate && __any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(flag, 1u);
+  }
   if (ds.P > 0) bulk_wait0();  // peer stores complete before the grid ends (made visible by the stream order)
   else bulk_wait_read0();
 }
@@ -649,13 +732,13 @@ inline bool make_tile_map(CUtensorMap *tm, const uint32_t *ptr, uint64_t rows, u
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ONE = false, bool DIRECT = false>
+template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ONE = false, bool DIRECT = false,
+          int IDB = 0>
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
-  // NT = 128 runs 32 keys per thread (same 4096-key tile, half the counter matrix per key)
-  constexpr int KPT = NT == 128 ? 32 : 16;
+  constexpr int KPT = 16;
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
-  constexpr int MINB = NT == 256 ? (KV ? 2 : 3) : (KV ? 3 : 4);
-  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE, DIRECT>;
+  constexpr int MINB = KV ? 2 : 3;
+  auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE, DIRECT, IDB>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
@@ -672,49 +755,48 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   CUtensorMap tmk, tmv;
   if (!make_tile_map(&tmk, a.keys, rows, Ly::T) || !make_tile_map(&tmv, KV ? a.vals : nullptr, rows, Ly::T))
     return cudaErrorInvalidValue;
-  const cudaError_t e = ONE ? launch_coop(k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals, a.G,
-                                          a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs, DistTarget{})
+  const cudaError_t e = ONE ? launch_coop(k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys, a.vals, a.ids,
+                                          a.flag, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs, DistTarget{})
                             : launch_ex(a.pdl != 0, k, dim3(grid), dim3(NT), smem, a.stream, tmk, tmv, a.keys,
-                                        a.vals, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs,
+                                        a.vals, a.ids, a.flag, a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs,
                                         a.ds ? *a.ds : DistTarget{});
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
-template <int KIND, bool KV, int LOGMP, int NT>
+template <int KIND, bool KV, int LOGMP, int IDB>
 inline cudaError_t k3v_launch_n(const K3pArgs &a) {
-  constexpr int STAGES = KV ? 1 : (LOGMP <= 3 && NT == 256 ? 3 : 2);  // m <= 8 key-only: 3 stages still fit 3 CTAs/SM
-  if constexpr (NT == 256) {
-    if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true>(a);
-  }
+  constexpr int NT = 256;
+  constexpr int STAGES = KV ? 1 : (LOGMP <= 3 ? 3 : 2);  // m <= 8 key-only: 3 stages still fit 3 CTAs/SM
+  if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true, false, IDB>(a);
   if (a.direct) {  // ablation: instantiated for the one-shift bucket kind only (SHIFT: DELTA with m*delta = 2^32)
-    if constexpr (NT == 256 && KIND == SHIFT) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, true>(a);
+    if constexpr (KIND == SHIFT) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, true>(a);
     return cudaErrorNotSupported;
   }
-  return a.ranged ? k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true>(a)
-                  : k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false>(a);
+  return a.ranged ? k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, false, false, IDB>(a)
+                  : k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, false, IDB>(a);
 }
 
-template <int KIND, bool KV, int LOGMP>
-inline cudaError_t k3v_launch_l(const K3pArgs &a) {
-  return a.nt == 128 ? k3v_launch_n<KIND, KV, LOGMP, 128>(a) : k3v_launch_n<KIND, KV, LOGMP, 256>(a);
-}
-
-template <int KIND, bool KV>
+template <int KIND, bool KV, int IDB>
 inline cudaError_t k3v_launch_kv(const K3pArgs &a) {
   uint32_t l = 1;
   while ((1u << l) < a.m) ++l;
   switch (l) {
-    case 1: return k3v_launch_l<KIND, KV, 1>(a);
-    case 2: return k3v_launch_l<KIND, KV, 2>(a);
-    case 3: return k3v_launch_l<KIND, KV, 3>(a);
-    case 4: return k3v_launch_l<KIND, KV, 4>(a);
-    default: return k3v_launch_l<KIND, KV, 5>(a);
+    case 1: return k3v_launch_n<KIND, KV, 1, IDB>(a);
+    case 2: return k3v_launch_n<KIND, KV, 2, IDB>(a);
+    case 3: return k3v_launch_n<KIND, KV, 3, IDB>(a);
+    case 4: return k3v_launch_n<KIND, KV, 4, IDB>(a);
+    default: return k3v_launch_n<KIND, KV, 5, IDB>(a);
   }
 }
 
 template <int KIND>
 inline cudaError_t k3v_launch(const K3pArgs &a) {
-  return a.vals ? k3v_launch_kv<KIND, true>(a) : k3v_launch_kv<KIND, false>(a);
+  if constexpr (KIND == IDS) {
+    if (a.id_bytes == 1) return a.vals ? k3v_launch_kv<KIND, true, 1>(a) : k3v_launch_kv<KIND, false, 1>(a);
+    return a.vals ? k3v_launch_kv<KIND, true, 4>(a) : k3v_launch_kv<KIND, false, 4>(a);
+  } else {
+    return a.vals ? k3v_launch_kv<KIND, true, 0>(a) : k3v_launch_kv<KIND, false, 0>(a);
+  }
 }
 
 }  // namespace ms

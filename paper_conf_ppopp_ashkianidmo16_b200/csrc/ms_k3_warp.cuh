@@ -22,7 +22,7 @@ namespace ms {
 // the tile's bucket starts S_t then give each key its shared-memory slot
 // (Eq. (2) one level down).  Keys (and values) arrive by one TMA
 // bulk copy per array (UBLKCP) on an mbarrier.
-template <int KIND, bool KV, int R, int LOGM, bool FULL, bool MATCH>
+template <int KIND, bool KV, int R, int LOGM, bool FULL>
 __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
                                         uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
                                         uint64_t base, uint32_t nt, const BucketParams &p,
@@ -62,13 +62,7 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
     // one shifted copy of the id feeds both the vote predicate (its sign) and
     // the sign-extension, and one LOP3 accumulates the difference mask
     uint32_t peers;
-    if constexpr (MATCH) {
-      // one MATCH.ANY per round: it runs on the ADU pipe, so its latency
-      // overlaps other warps' work and costs one issue slot instead of the
-      // ~5 per id bit of the ballot form (invalid lanes, id = ~0, form a
-      // group of their own)
-      peers = __match_any_sync(0xFFFFFFFFu, id);
-    } else {
+    {
       uint32_t diff = FULL ? 0u : ~__ballot_sync(0xFFFFFFFFu, valid);
 #pragma unroll
       for (int b = 0; b < LOGM; ++b) {
@@ -159,7 +153,7 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
   }
 }
 
-template <int KIND, bool KV, int R, int LOGM, bool MATCH>
+template <int KIND, bool KV, int R, int LOGM>
 __global__ void __launch_bounds__(kThreads)
 k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
             const void *__restrict__ ids, const uint32_t *__restrict__ G,
@@ -177,7 +171,7 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   __shared__ uint32_t wsum[kWarps];
 
   const uint32_t tid = threadIdx.x;
-  const uint32_t tile = p.reverse ? L - 1 - blockIdx.x : blockIdx.x;  // reverse: L2 reuse of K1's tail
+  const uint32_t tile = blockIdx.x;
   const uint64_t base = (uint64_t)tile * T;
   const uint32_t nt = (uint32_t)umin64(T, n - base);
   const bool full = (nt == T);
@@ -209,10 +203,10 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   __syncthreads();
   if (full) {
     mbar_wait(&bar, 0);
-    k3_tile<KIND, KV, R, LOGM, true, MATCH>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+    k3_tile<KIND, KV, R, LOGM, true>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
                                spl_s, id8_s, wsum, gcol);
   } else {
-    k3_tile<KIND, KV, R, LOGM, false, MATCH>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+    k3_tile<KIND, KV, R, LOGM, false>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
                                 spl_s, id8_s, wsum, gcol);
   }
 }
@@ -226,10 +220,9 @@ inline size_t k3w_smem(int R, bool kv, bool id8) {
 template <int KIND, bool KV, int R, int LOGM>
 inline cudaError_t k3w_launch_l(const K3pArgs &a) {
   constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC && KIND != SHIFT);
-  // ballot ranks; MS_K3W_MATCH=1 selects __match_any_sync (measured 1.6x slower
-  // at m = 256 on B200: MATCH.ANY is ADU-bound)
-  static const bool match = getenv("MS_K3W_MATCH") && atoi(getenv("MS_K3W_MATCH"));
-  auto k = match ? k3_postscan<KIND, KV, R, LOGM, true> : k3_postscan<KIND, KV, R, LOGM, false>;
+  // ballot ranks (__match_any_sync measured 1.6x slower at m = 256 on B200: MATCH.ANY is
+  // ADU-bound)
+  auto k = k3_postscan<KIND, KV, R, LOGM>;
   const size_t smem = k3w_smem(R, KV, id8);
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(a.L), dim3(kThreads), smem, a.stream, a.keys, a.vals, a.ids,

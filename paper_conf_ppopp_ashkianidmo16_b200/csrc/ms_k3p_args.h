@@ -13,7 +13,6 @@ namespace ms {
 
 // Ranged variant with the range scan folded into K3 (range_base below):
 // HC = K1r's R = C*k sub-range rows of m counts; offsets written by CTA 0.
-// HC == nullptr: K3 reads GB[c][:] written by K2r instead.
 struct RangeScan {
   const uint32_t *HC;
   uint32_t *offsets;
@@ -41,16 +40,17 @@ struct K3pArgs {
   const uint32_t *G;
   uint32_t *keys_out, *vals_out;
   uint32_t n, L, m, id_bytes, kpt;
-  uint32_t nt;              // K3p threads per CTA (128 or 256); tile = nt * 16 keys
+  uint32_t nt;              // K3 v2 threads per CTA (256); tile = nt * 16 keys
   const BucketParams *bp;  // host copy, passed by value to the kernel
   int sms;
   cudaStream_t stream;
   int ranged = 0;               // 1: CTA-range mode (G = GB[C][m], ms_ranged.cuh); 2: one cooperative launch; m <= 32
   int pdl = 0;                  // 1: programmatic dependent launch after K2 (ms_device.cuh pdl_wait)
   uint32_t *grid_out = nullptr;  // non-null: only compute the grid C (no launch)
-  RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged: fold K2r into K3's prologue when rs.HC is set
+  RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged / ONE: the range scan's input (K3's prologue)
   const DistTarget *ds = nullptr;           // fused sharded scatter (K3 v2, tile variant only)
-  int direct = 0;                           // ablation: K3 v2 without the local reorder (MS_K3_DIRECT=1)
+  int direct = 0;                           // ablation: K3 v2 without the local reorder (MS_ABLATION_DIRECT)
+  uint32_t *flag = nullptr;                 // IDS + validation: set to 1 when some id >= m
 };
 
 // Launch with cudaLaunchAttributeProgrammaticStreamSerialization when `pdl`:
@@ -72,9 +72,9 @@ inline cudaError_t launch_ex(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 b
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
-// ============================================================== K2r folded into K3
+// ============================================================== range scan folded into K3
 // Terms 1+2 of Eq. (2) for range c, computed redundantly by every K3 CTA from
-// K1r's rows (replaces the K2r launch and its hand-off; the R x m words are
+// K1r's rows (no separate scan launch or hand-off; the R x m words are
 // L2-resident, R*m*4 <= 76 KB for m <= 16):
 //   pre_j = sum_{r < c*k} HC[r][j],  tot_j = sum_r HC[r][j],
 //   GB[c][j] = sum_{i<j} tot_i + pre_j,  offsets[j] = sum_{i<j} tot_i (CTA 0).
@@ -200,24 +200,13 @@ inline cudaError_t launch_coop(void (*kern)(KArgs...), dim3 grid, dim3 block, si
 
 constexpr uint32_t kMaxRanges = 1024;  // upper bound on the CTA-range count C (workspace sizing)
 
-cudaError_t k3p_launch_lowbits(const K3pArgs &a);
-cudaError_t k3p_launch_shiftc(const K3pArgs &a);
-cudaError_t k3p_launch_shift(const K3pArgs &a);
-cudaError_t k3p_launch_delta(const K3pArgs &a);
-cudaError_t k3p_launch_splitters(const K3pArgs &a);
-cudaError_t k3p_launch_ids(const K3pArgs &a);
-// m <= 32, second generation (ms_k3_v2.cuh): TMA-tensor staging, keys in registers
+// m <= 32 (ms_k3_v2.cuh): TMA-tensor staging, keys in registers, blocked private counters
 cudaError_t k3v_launch_lowbits(const K3pArgs &a);
 cudaError_t k3v_launch_shiftc(const K3pArgs &a);
 cudaError_t k3v_launch_shift(const K3pArgs &a);
 cudaError_t k3v_launch_delta(const K3pArgs &a);
 cudaError_t k3v_launch_splitters(const K3pArgs &a);
-// 32 < m <= 256, kinds other than MS_IDS: two-digit LSD local multisplit (ms_k3_lsd.cuh)
-cudaError_t k3h_launch_lowbits(const K3pArgs &a);
-cudaError_t k3h_launch_shiftc(const K3pArgs &a);
-cudaError_t k3h_launch_shift(const K3pArgs &a);
-cudaError_t k3h_launch_delta(const K3pArgs &a);
-cudaError_t k3h_launch_splitters(const K3pArgs &a);
+cudaError_t k3v_launch_ids(const K3pArgs &a);
 // m > 32: warp-ballot K3 (ms_k3_warp.cuh); kpt carries the rounds per warp R (8 or 16)
 cudaError_t k3w_launch_lowbits(const K3pArgs &a);
 cudaError_t k3w_launch_shiftc(const K3pArgs &a);

@@ -1,4 +1,4 @@
-// ms_ranged.cuh -- the CTA-range form of Eq. (2): K1r range histograms, K2r range scan (sm_100a).
+// ms_ranged.cuh -- the CTA-range form of Eq. (2): K1r range histograms (sm_100a).
 //
 // Eq. (2) holds for ANY partition of the input into
 // consecutive subproblems.  The tile variant (ms_kernels.cuh) uses one
@@ -6,12 +6,12 @@
 // subproblems are the C contiguous tile RANGES that the C persistent K3 CTAs
 // own (range c = tiles [c*L/C, (c+1)*L/C), C = K3's resident grid, <= ~900):
 //   K1r: HC[c][j] = #{keys of range c in bucket j}      (local step 1 of the range)
-//   K2r: GB[c][j] = sum_{k<j} total_k + sum_{c'<c} HC[c'][j]   (terms 1+2 of Eq. 2)
-//   K3 : walks its range's tiles in order and keeps G_j for the current tile
+//   K3 prologue (range_base, ms_k3p_args.h): GB[c][j] = sum_{k<j} total_k + sum_{c'<c} HC[c'][j]
+//        (terms 1+2 of Eq. 2), then K3 walks its range's tiles in order and keeps G_j for the current tile
 //        as a running sum in registers (GB[c][j] + counts of the range's earlier
 //        tiles), i.e. Eq. (2) once more one level down, with no H/G array.
 // H/G traffic drops from 16 m / T bytes per key to 16 m C / n, and K2 becomes a
-// one-CTA scan of C x m words instead of a grid-wide chained scan of m x L.
+// scan of C x m words folded into K3's prologue instead of a grid-wide chained scan of m x L.
 // Stable by construction: ranges, tiles and keys are all visited in input order.
 #pragma once
 #include "ms_k3p_args.h"
@@ -80,7 +80,7 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   uint64_t k0, k1;
   range_span(blockIdx.x / k, blockIdx.x % k, k, C, L, T, n, &k0, &k1);
 
-  pdl_trigger();  // K2r (launched with PDL) may be scheduled once every K1r CTA has started
+  pdl_trigger();  // K3 (launched with PDL) may be scheduled once every K1r CTA has started
   uint4 *c4 = reinterpret_cast<uint4 *>(c8);
   for (uint32_t i = tid; i < m * (NT1 / 16); i += NT1) c4[i] = make_uint4(0, 0, 0, 0);
   if (tid < 32) acc[tid] = 0;
@@ -178,60 +178,7 @@ inline size_t k1r_smem(uint32_t m, int kind, int nt1) {
   return (kind == SPLITTERS ? (kMaxM + kSplBins) * 4 : 0) + 32 * 4 + (size_t)m * nt1;
 }
 
-// ============================================================== K2r
-// One CTA over the R = C*k sub-range rows (staged in shared memory by one
-// coalesced sweep, so nothing below waits on a chain of global loads):
-// GB[c][j] = start_j + sum_{r < c*k} HC[r][j] with start_j = sum_{i<j} total_i
-// (Eq. (2) terms 1+2 over ranges), offsets[j] = start_j, offsets[m] = n.
-// Thread (s, j) (j = tid mod MP, s = tid / MP) owns the rows of segment s:
-// segment sums -> inclusive scan over segments per bucket -> bucket starts ->
-// rescan of the segment emitting GB at every range's first row.
-constexpr int kR2Threads = 1024;
-constexpr uint32_t kMaxRangeRows = 1280;  // R <= max(C, 8 * SMs) on B200 (<= 1184)
-
-__global__ void __launch_bounds__(kR2Threads)
-k2r_scan(const uint32_t *__restrict__ HC, uint32_t *__restrict__ GB, uint32_t R, uint32_t k, uint32_t m,
-         uint32_t logmp, uint32_t *__restrict__ offsets, uint32_t n) {
-  extern __shared__ uint32_t hs[];  // [R][m]
-  __shared__ uint32_t seg[kR2Threads];
-  __shared__ uint32_t start[32];
-  const uint32_t tid = threadIdx.x;
-  const uint32_t words = R * m;
-  pdl_wait();  // K1r's HC rows are complete and visible
-  pdl_trigger();
-  for (uint32_t i = tid; i < words; i += kR2Threads) hs[i] = HC[i];
-  __syncthreads();
-  const uint32_t MP = 1u << logmp, j = tid & (MP - 1), s = tid >> logmp, NS = kR2Threads >> logmp;
-  const uint32_t r0 = (uint32_t)((uint64_t)s * R / NS), r1 = (uint32_t)((uint64_t)(s + 1) * R / NS);
-  uint32_t sum = 0;
-  if (j < m)
-    for (uint32_t r = r0; r < r1; ++r) sum += hs[r * m + j];
-  seg[tid] = sum;
-  __syncthreads();
-  // inclusive scan over s for each j (stride MP in seg), Hillis-Steele
-  for (uint32_t d = 1; d < NS; d <<= 1) {
-    const uint32_t add = s >= d ? seg[tid - (d << logmp)] : 0u;
-    __syncthreads();
-    seg[tid] += add;
-    __syncthreads();
-  }
-  if (tid < 32) {  // bucket starts: exclusive scan of the column totals (m <= 32)
-    const uint32_t tot = tid < m ? seg[((NS - 1) << logmp) + tid] : 0u;
-    const uint32_t incl = warp_incl_scan(tot, tid);
-    start[tid] = incl - tot;
-    if (offsets != nullptr) {
-      if (tid < m) offsets[tid] = incl - tot;
-      if (tid == 0) offsets[m] = n;
-    }
-  }
-  __syncthreads();
-  if (j < m) {
-    uint32_t run = start[j] + seg[tid] - sum;  // exclusive over earlier segments
-    for (uint32_t r = r0; r < r1; ++r) {
-      if (r % k == 0) GB[(r / k) * m + j] = run;
-      run += hs[r * m + j];
-    }
-  }
-}
+// Rows of K1r's range-count matrix: R = C * k <= max(C, 8 * SMs) on B200 (<= 1184).
+constexpr uint32_t kMaxRangeRows = 1280;
 
 }  // namespace ms

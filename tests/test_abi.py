@@ -28,10 +28,10 @@ def test_exports_every_declared_symbol():
     assert set(names) == set(_abi.EXPORTS)
 
 
-def _create(spec: BucketSpec, max_n=1 << 20, kv=0, flags=0):
+def _create(spec: BucketSpec, max_n=1 << 20, kv=0, flags=0, device=-1):
     h = ctypes.c_void_p()
     c = spec._c()
-    st = _abi.lib().ms_plan_create(ctypes.byref(h), ctypes.byref(c), max_n, kv, flags)
+    st = _abi.lib().ms_plan_create(ctypes.byref(h), ctypes.byref(c), max_n, kv, flags, device)
     return st, h
 
 
@@ -44,6 +44,9 @@ def _create(spec: BucketSpec, max_n=1 << 20, kv=0, flags=0):
     (BucketSpec("splitters", 3, splitters=[5, 4]), 0),   # not non-decreasing
     (BucketSpec("ids", 8, id_bytes=2), 0),
     (BucketSpec("delta", 8, delta=5), 2 | 4),      # two variants forced
+    (BucketSpec("delta", 8, delta=5), 4 | 8),
+    (BucketSpec("delta", 8, delta=5), 2 | 8),
+    (BucketSpec("delta", 8, delta=1 << 29), 16 | 2),  # ablation + forced variant
     (BucketSpec("delta", 8, delta=5), 64),         # unknown flag
 ])
 def test_plan_create_rejects(spec, flags):
@@ -64,6 +67,51 @@ def test_plan_create_accepts(spec):
     st, h = _create(spec)
     assert st == _abi.MS_OK and h.value
     _abi.lib().ms_plan_destroy(h)
+
+
+@pytest.mark.parametrize("spec,flags", [
+    (BucketSpec("delta", 64, delta=1 << 26), 4),   # ranged / ONE need m <= 32
+    (BucketSpec("delta", 64, delta=1 << 26), 8),
+    (BucketSpec("delta", 8, delta=5), 16),         # Direct ablation: DELTA with m * delta = 2^32 only
+    (BucketSpec("delta", 64, delta=1 << 26), 16),
+    (BucketSpec("ids", 8), 16),
+])
+def test_plan_create_unsupported(spec, flags):
+    st, h = _create(spec, flags=flags)
+    assert st == _abi.MS_ERR_UNSUPPORTED and not h.value
+
+
+def test_plan_create_device_argument():
+    assert _create(BucketSpec("delta", 8, delta=5), device=-2)[0] == _abi.MS_ERR_INVALID_ARG
+    st, h = _create(BucketSpec("delta", 8, delta=5), device=0)
+    assert st == _abi.MS_OK
+    _abi.lib().ms_plan_destroy(h)
+
+
+def _variant(spec, n, kv, flags=0):
+    st, h = _create(spec, max_n=1 << 28, kv=kv, flags=flags)
+    assert st == _abi.MS_OK
+    v = ctypes.c_int32()
+    assert _abi.lib().ms_plan_geometry(h, n, None, None, ctypes.byref(v)) == _abi.MS_OK
+    _abi.lib().ms_plan_destroy(h)
+    return v.value
+
+
+def test_variant_rule():
+    """ms_plan_geometry reports the variant the run takes: ONE for key-only m <= 32 and
+    for key-value up to 64 tiles per SM, then ranged (m <= 16) or tile (m > 16); tile for m > 32;
+    a MS_VARIANT_* flag always wins.  (Without a GPU the SM count is B200's 148.)"""
+    T, ONE, RANGED, TILE = _abi.VARIANT_TILE, _abi.VARIANT_ONE, _abi.VARIANT_RANGED, _abi.VARIANT_TILE
+    d8, d32, d256 = (BucketSpec("delta", 8, delta=1 << 29), BucketSpec("delta", 32, delta=1 << 27),
+                     BucketSpec("delta", 256, delta=1 << 24))
+    assert _variant(d8, 1 << 28, 0) == ONE and _variant(d32, 1 << 28, 0) == ONE
+    assert _variant(d8, 1 << 25, 1) == ONE and _variant(d32, 1 << 25, 1) == ONE   # 8192 tiles <= 64 * 148
+    assert _variant(d8, 1 << 28, 1) == RANGED and _variant(d32, 1 << 28, 1) == TILE
+    assert _variant(BucketSpec("ids", 16), 1 << 28, 1) == RANGED
+    assert _variant(d256, 1 << 20, 0) == T and _variant(d256, 1 << 28, 1) == T
+    for flags, want in ((2, TILE), (4, RANGED), (8, ONE)):
+        assert _variant(d8, 1 << 28, 1, flags) == want and _variant(d32, 1000, 0, flags) == want
+    assert _variant(d8, 1 << 20, 0, 16) == TILE      # the Direct ablation runs the tile variant
 
 
 def test_geometry_and_workspace():

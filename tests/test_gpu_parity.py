@@ -21,14 +21,29 @@ def _pkg():
     return P
 
 
-def _run_case(case, variant=None, want_offsets=True):
+FORCED = {"3k": 0, "tile": 0, "direct": 0, "ranged": 1, "one": 2}
+
+
+def _run_case(case, variant=None, want_offsets=True, expect_variant=None):
+    """Runs the case through ms_run and checks that the kernels which ran are the ones the
+    variant names: ms_plan_last_launches must equal the launch count of the variant the plan
+    reports (or was forced to), so a silent re-routing to another path fails the test."""
     P = _pkg()
+    from paper_conf_ppopp_ashkianidmo16_b200 import _abi
     spec = P.BucketSpec(**case["spec_kw"])
     n = len(case["keys"])
-    plan = P.Plan(spec, max(n, 1), with_values=case["vals"] is not None, variant=variant)
+    kv = case["vals"] is not None
+    plan = P.Plan(spec, max(n, 1), with_values=kv, variant=variant)
     ko, vo, off = plan.run(to_dev(case["keys"]), to_dev(case["vals"]), to_dev(case["ids"]),
                            want_offsets=want_offsets)
     torch.cuda.synchronize()
+    v = plan.geometry(n)[2]
+    if variant is not None:
+        assert v == FORCED[variant], f"geometry reports variant {v} for forced {variant}"
+    if expect_variant is not None:
+        assert v == expect_variant, f"variant {v}, expected {expect_variant}"
+    assert plan.last_launches() == (_abi.LAUNCHES[v] if n else 0), \
+        f"{plan.last_launches()} launches for variant {v} (n={n})"
     return from_dev(ko), from_dev(vo), (None if off is None else from_dev(off)), plan
 
 
@@ -51,53 +66,53 @@ MS = [1, 2, 3, 5, 8, 31, 32, 33, 64, 127, 255, 256]
 
 
 # Low-bit buckets need a power-of-two m (reading #10); m > 32 always uses the tile variant, so the
-# forced CTA-range variant is only generated for m <= 32.
-MATRIX = [(kind, m, variant) for variant in (None, "ranged") for kind in ("lowbits", "delta", "splitters", "ids")
-          for m in MS if not (kind == "lowbits" and m & (m - 1)) and not (variant == "ranged" and m > 32)]
+# forced CTA-range and ONE variants are only generated for m <= 32.
+MATRIX = [(kind, m, variant) for variant in (None, "3k", "ranged", "one")
+          for kind in ("lowbits", "delta", "splitters", "ids")
+          for m in MS if not (kind == "lowbits" and m & (m - 1)) and not (variant in ("ranged", "one") and m > 32)]
 
 
 @pytest.mark.parametrize("kind,m,variant", MATRIX)
 def test_parity_matrix(kind, m, variant):
-    """kind x m x n (empty, ragged, tile edges) x KO/KV, uniform keys; the default
-    variant (tile at these sizes) and the forced CTA-range variant (m <= 32)."""
+    """kind x m x n (empty, ragged, tile edges) x KO/KV, uniform keys; the default variant
+    (ONE for m <= 32 at these sizes, tile above) and every forced variant, each run asserting
+    the number of kernels it launched."""
     for i, n in enumerate(NS):
         for kv in (False, True):
             case = make_case(kind, m, n, seed=1000 * m + i, kv=kv, id_bytes=1 if i % 2 else 4)
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} n={n} kv={kv} {variant}")
 
 
-@pytest.mark.parametrize("k2r", [False, True])
+@pytest.mark.parametrize("variant", ["ranged", "one"])
 @pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("ids", 5, True),
-                                       ("lowbits", 2, False), ("delta", 32, True), ("delta", 16, True)])
-def test_ranged_range_edges(kind, m, kv, k2r, monkeypatch):
-    """Ranged variant around C = resident K3 CTAs: L < C, L = C +- 1, L = 3C + r (ranges of 1..4 tiles,
-    the ragged last tile at the end of the last range); the range scan folded into K3's prologue
-    (default) and as a separate K2r launch (MS_RANGED_K2=1)."""
-    if k2r:
-        monkeypatch.setenv("MS_RANGED_K2", "1")
-    P = _pkg()
-    probe = P.Plan(P.BucketSpec(**make_case(kind, m, 1, 0, kv=kv)["spec_kw"]), 1 << 24, with_values=kv,
-                   variant="ranged")
-    T, _, v = probe.geometry(1 << 24)
-    assert v == 1
+                                       ("lowbits", 2, False), ("delta", 32, True), ("delta", 16, True),
+                                       ("ids", 32, False)])
+def test_ranged_range_edges(kind, m, kv, variant):
+    """CTA-range (K1r -> K3, 2 launches) and ONE (1 launch) variants around C = resident K3 CTAs:
+    L < C, L = C +- 1, L = 3C + r (ranges of 1..4 tiles, the ragged last tile at the end of the
+    last range); every run asserts its launch count."""
+    T = 4096
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     for i, L in enumerate([sms - 1, 2 * sms, 4 * sms + 1, 6 * sms - 1, 6 * sms, 6 * sms + 1, 13 * sms + 7]):
         for n in (L * T, L * T - T + 3):
             case = make_case(kind, m, n, seed=77 + i, kv=kv)
-            _assert_equal(case, _run_case(case, "ranged"), _expect(case), f"{kind} m={m} L={L} n={n}")
+            _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} L={L} n={n} {variant}")
 
 
-@pytest.mark.parametrize("kind,m", [(k, m) for k in ("lowbits", "delta", "splitters") for m in (33, 64, 127, 256)
-                                    if not (k == "lowbits" and m & (m - 1))])
-def test_parity_two_digit_k3(kind, m, monkeypatch):
-    """The two-digit (LSD 16 x 16) K3 for m > 32, an ablation kept behind MS_K3H=1: bit-exact on ragged
-    sizes, skewed buckets and a multi-wave n."""
-    monkeypatch.setenv("MS_K3H", "1")
-    for i, (n, dist) in enumerate([(1, "uniform"), (4095, "uniform"), (4097, "hot"), (100003, "binomial"),
-                                   ((1 << 22) + 5, "uniform")]):
-        for kv in (False, True):
-            case = make_case(kind, m, n, seed=300 + 10 * m + i, dist=dist, kv=kv)
-            _assert_equal(case, _run_case(case), _expect(case), f"k3h {kind} m={m} n={n} {dist} kv={kv}")
+@pytest.mark.parametrize("n", [(1 << 26) + 5, 1 << 28])
+@pytest.mark.parametrize("kind,m", [("delta", 2), ("delta", 8), ("lowbits", 16), ("splitters", 16), ("ids", 8),
+                                    ("delta", 32), ("ids", 32)])
+def test_parity_default_large_kv(kind, m, n):
+    """The library's DEFAULT key-value path above 64 tiles per SM: K1r -> K3 (2 launches) for
+    m <= 16, K1 -> K2 -> K3 (3 launches) for 16 < m <= 32 -- at n = 2^26 + 5 and 2^28, full compare."""
+    case = make_case(kind, m, n, seed=900 + m, kv=True, vals_kind="random")
+    want = _abi_mod().VARIANT_RANGED if m <= 16 else _abi_mod().VARIANT_TILE
+    _assert_equal(case, _run_case(case, expect_variant=want), _expect(case), f"default KV {kind} m={m} n={n}")
+
+
+def _abi_mod():
+    from paper_conf_ppopp_ashkianidmo16_b200 import _abi
+    return _abi
 
 
 @pytest.mark.parametrize("kv", [False, True])
@@ -118,13 +133,13 @@ def test_parity_distributions(kind, m, dist):
     """Skewed workloads (§6.5): binomial, 75 % hot bucket, all in one bucket."""
     for n in (4097, (1 << 20) + 7):
         case = make_case(kind, m, n, seed=7 + m, dist=dist, kv=True)
-        for variant in ([None, "ranged"] if m <= 32 else [None]):
+        for variant in ([None, "3k", "ranged", "one"] if m <= 32 else [None, "3k"]):
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} {dist} n={n} {variant}")
 
 
-@pytest.mark.parametrize("variant", [None, "3k", "ranged"])
+@pytest.mark.parametrize("variant", [None, "3k", "ranged", "one"])
 @pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("lowbits", 32, True),
-                                       ("lowbits", 2, True)])
+                                       ("lowbits", 2, True), ("ids", 32, False), ("ids", 16, True)])
 def test_parity_2p25(kind, m, kv, variant):
     """BJ configs C2 / C3 size (n = 2^25), full element-wise compare, every variant."""
     case = make_case(kind, m, 1 << 25, seed=W.SEEDS["C3"], kv=kv, vals_kind="random")
@@ -382,12 +397,11 @@ def test_fused_scatter_rejects_unsupported():
 
 
 @pytest.mark.parametrize("m", [2, 8, 32])
-def test_parity_direct_ablation(m, monkeypatch):
-    """The Direct (no local reorder) K3 ablation, MS_K3_DIRECT=1 (SHIFT bucket kind: DELTA with
-    m * delta = 2^32), bit-exact on ragged sizes, KO and KV."""
-    monkeypatch.setenv("MS_K3_DIRECT", "1")
+def test_parity_direct_ablation(m):
+    """The Direct (no local reorder) K3 ablation, MS_ABLATION_DIRECT (SHIFT bucket kind: DELTA with
+    m * delta = 2^32), bit-exact on ragged sizes, KO and KV (3 launches: K1, K2, Direct K3)."""
     for i, n in enumerate([1, 4095, 4097, 100003, (1 << 21) + 3]):
         for kv in (False, True):
             case = make_case("delta", m, n, seed=2 * (400 + i), kv=kv)  # even seed: delta = 2^32 / m
             assert case["spec_kw"]["delta"] == (1 << 32) // m
-            _assert_equal(case, _run_case(case), _expect(case), f"direct m={m} n={n} kv={kv}")
+            _assert_equal(case, _run_case(case, "direct"), _expect(case), f"direct m={m} n={n} kv={kv}")
