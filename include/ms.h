@@ -175,6 +175,10 @@ ms_status ms_plan_check(ms_plan_t plan, void *workspace, void *stream);
 ms_status ms_plan_destroy(ms_plan_t plan);
 const char *ms_status_string(ms_status s);
 
+/* The plan's bucket spec (splitters reported as NULL) and whether it plans
+ * key-value runs (host only). */
+ms_status ms_plan_spec(ms_plan_t plan, ms_bucket_spec *spec, int32_t *with_values);
+
 /* Number of kernel launches the last ms_run / ms_run_host on this plan
  * enqueued (for the bench's gpu_launches claim). */
 int32_t ms_plan_last_launches(ms_plan_t plan);
@@ -274,6 +278,51 @@ typedef struct {
 
 ms_status ms_dist_targets(int32_t nranks, int32_t rank, uint32_t m, const uint64_t *counts, uint64_t *delta,
                           uint64_t *win_start);
+
+/* ---------------------------------------------------------------------------
+ * ms_dist_run -- the sharded stable multisplit as ONE collective call per rank
+ * over an NCCL communicator (Eq. (2), with the
+ * ranks as the outermost subproblems, the hierarchical split of P:667-674):
+ *   1. local stable multisplit of this rank's shard (ms_run) into staging
+ *      buffers inside `workspace`;
+ *   2. NCCL all-gather of the P x m per-rank bucket counts (u64), computed on
+ *      the device from the local offsets; the count matrix is copied to the
+ *      host -- the ONE point where the call synchronises `stream` (the piece
+ *      sizes are host arguments of the NCCL point-to-point calls);
+ *   3. ms_dist_pieces (above): global bucket starts, this rank's balanced
+ *      window [win_start, win_start + win_len) and its <= m+P-1 pieces;
+ *   4. one NCCL group of send/recv over NVLink/NVSwitch (pieces to self by
+ *      device copies) landing every piece at its final offset in the owner's
+ *      window -- no receive-side permutation.
+ * Every rank calls it with the same plan spec; rank and P come from `comm`
+ * (an ncclComm_t, e.g. from ms_nccl_comm_init), whose device the call runs on.
+ * keys_in/vals_in/ids: this rank's shard (n_local elements, device); keys_out
+ * / vals_out: this rank's window buffers of out_capacity elements (device; the
+ * window length is at most ceil(N/P) for N = total elements), written in
+ * [0, win_len).  offsets_global (HOST, m+1 u64, or NULL): global bucket
+ * starts; win_start / win_len (HOST, or NULL).  The output is complete when
+ * `stream` completes; the concatenation of the windows over ranks is the
+ * single-GPU stable multisplit of the concatenated shards (rank order).
+ * Workspace: ms_dist_workspace_size.  Errors: argument errors as ms_run, plus
+ * MS_ERR_INVALID_ARG if the window exceeds out_capacity (checked after the
+ * count exchange, before any data moves) and MS_ERR_NCCL if NCCL cannot be
+ * loaded (libnccl.so.2, dlopen'ed at first use) or a call fails.
+ * ------------------------------------------------------------------------- */
+ms_status ms_dist_workspace_size(ms_plan_t plan, uint64_t n_local, int32_t nranks, size_t *bytes);
+ms_status ms_dist_run(ms_plan_t plan, void *nccl_comm, const uint32_t *keys_in, const uint32_t *vals_in,
+                      const void *ids, uint64_t n_local, uint32_t *keys_out, uint32_t *vals_out,
+                      uint64_t out_capacity, uint64_t *offsets_global, uint64_t *win_start, uint64_t *win_len,
+                      void *workspace, size_t workspace_bytes, void *stream);
+
+/* NCCL bootstrap for ms_dist_run (the 128-byte unique id travels between the
+ * processes by any means, e.g. a torch.distributed broadcast):
+ * ms_nccl_get_unique_id writes NCCL_UNIQUE_ID_BYTES (128) bytes to `id` (rank 0);
+ * ms_nccl_comm_init makes `device` current and creates rank `rank` of an
+ * nranks-rank communicator (*comm = the ncclComm_t); ms_nccl_comm_destroy
+ * frees it.  MS_ERR_NCCL if NCCL cannot be loaded or fails. */
+ms_status ms_nccl_get_unique_id(void *id);
+ms_status ms_nccl_comm_init(void **comm, int32_t nranks, int32_t rank, const void *id, int device);
+ms_status ms_nccl_comm_destroy(void *comm);
 ms_status ms_postscan_scatter(ms_plan_t plan, const uint32_t *keys_in, const uint32_t *vals_in,
                               const uint32_t *G, uint64_t n, const ms_scatter_target *target, void *workspace,
                               size_t workspace_bytes, void *stream);

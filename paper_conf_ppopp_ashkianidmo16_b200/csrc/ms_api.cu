@@ -408,6 +408,13 @@ ms_status ms_plan_geometry(ms_plan_t p, uint64_t n, uint32_t *tile, uint64_t *nu
 
 int32_t ms_plan_last_launches(ms_plan_t p) { return p ? p->last_launches : -1; }
 
+ms_status ms_plan_spec(ms_plan_t p, ms_bucket_spec *spec, int32_t *with_values) {
+  if (!p) return MS_ERR_INVALID_ARG;
+  if (spec) *spec = p->spec;  // splitters: NULL (the plan keeps its own copy)
+  if (with_values) *with_values = p->kv;
+  return MS_OK;
+}
+
 ms_status ms_plan_trace(ms_plan_t p, int enable) {
   if (!p) return MS_ERR_INVALID_ARG;
   if (enable) p->trace_runs = 0;

@@ -107,3 +107,229 @@ extern "C" ms_status ms_dist_targets(int32_t P, int32_t rank, uint32_t m, const 
   for (int32_t r = 0; r <= P; ++r) win_start[r] = W.start(r);
   return MS_OK;
 }
+
+// =========================================================================
+// ms_dist_run: the sharded multisplit as ONE stream-ordered collective call
+// over an NCCL communicator.  Eq. (2) with the ranks
+// as the outermost subproblems (hierarchical split P:667-674):
+//   1. local stable multisplit of the shard (ms_run) into staging buffers
+//      carved from the workspace; its m+1 local offsets;
+//   2. counts h_g[b] = off[b+1] - off[b] (u64, device), NCCL all-gather of the
+//      P x m count matrix, copied to the host (the ONE synchronisation: the
+//      piece sizes are host arguments of the point-to-point calls);
+//   3. ms_dist_pieces: global bucket starts, this rank's balanced window and
+//      the <= m+P-1 contiguous pieces it sends / the pieces it receives;
+//   4. one NCCL group of send/recv (pieces to self: device-to-device copies)
+//      landing every piece at its final offset in the owner's window.
+// NCCL is loaded at run time (dlopen of libnccl.so.2 -- the process's NCCL,
+// e.g. the one torch already loaded), so libms.so has no link-time NCCL
+// dependency and loads on machines without it.
+// =========================================================================
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <cstring>
+#include <mutex>
+
+namespace {
+
+struct Nccl {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId *);
+  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int);
+  ncclResult_t (*CommDestroy)(ncclComm_t);
+  ncclResult_t (*CommCount)(const ncclComm_t, int *);
+  ncclResult_t (*CommUserRank)(const ncclComm_t, int *);
+  ncclResult_t (*CommCuDevice)(const ncclComm_t, int *);
+  ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t);
+  ncclResult_t (*Send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
+  ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
+  ncclResult_t (*GroupStart)();
+  ncclResult_t (*GroupEnd)();
+};
+
+const Nccl &nccl() {
+  static Nccl N;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+    bool all = true;
+    auto sym = [&](auto &fn, const char *name) {
+      fn = reinterpret_cast<std::remove_reference_t<decltype(fn)>>(dlsym(h, name));
+      all = all && fn != nullptr;
+    };
+    sym(N.GetUniqueId, "ncclGetUniqueId");
+    sym(N.CommInitRank, "ncclCommInitRank");
+    sym(N.CommDestroy, "ncclCommDestroy");
+    sym(N.CommCount, "ncclCommCount");
+    sym(N.CommUserRank, "ncclCommUserRank");
+    sym(N.CommCuDevice, "ncclCommCuDevice");
+    sym(N.AllGather, "ncclAllGather");
+    sym(N.Send, "ncclSend");
+    sym(N.Recv, "ncclRecv");
+    sym(N.GroupStart, "ncclGroupStart");
+    sym(N.GroupEnd, "ncclGroupEnd");
+    N.ok = all;
+  });
+  return N;
+}
+
+constexpr size_t kDAlign = 256;
+inline size_t dalign(size_t x) { return (x + kDAlign - 1) / kDAlign * kDAlign; }
+
+// counts[b] = off[b+1] - off[b] as u64 (local bucket sizes of this rank's shard)
+__global__ void k_counts_from_offsets(const uint32_t *off, uint64_t *counts, uint32_t m) {
+  for (uint32_t b = threadIdx.x; b < m; b += blockDim.x) counts[b] = (uint64_t)(off[b + 1] - off[b]);
+}
+
+struct DistLayout {
+  size_t local_ws, off_keys, off_vals, off_loff, off_cnt, off_gath, bytes;
+};
+
+DistLayout dist_layout(ms_plan_t plan, uint32_t m, int kv, uint64_t n_local, int nranks, ms_status *st) {
+  DistLayout d{};
+  size_t ws = 0;
+  *st = ms_plan_workspace_size(plan, n_local, &ws);
+  d.local_ws = dalign(ws);
+  d.off_keys = d.local_ws;
+  d.off_vals = d.off_keys + dalign(n_local * 4);
+  d.off_loff = d.off_vals + (kv ? dalign(n_local * 4) : 0);
+  d.off_cnt = d.off_loff + dalign((size_t)(m + 1) * 4);
+  d.off_gath = d.off_cnt + dalign((size_t)m * 8);
+  d.bytes = d.off_gath + dalign((size_t)nranks * m * 8);
+  return d;
+}
+
+}  // namespace
+
+extern "C" ms_status ms_nccl_get_unique_id(void *id) {
+  if (!id) return MS_ERR_INVALID_ARG;
+  const Nccl &N = nccl();
+  if (!N.ok) return MS_ERR_NCCL;
+  ncclUniqueId u;
+  if (N.GetUniqueId(&u) != ncclSuccess) return MS_ERR_NCCL;
+  memcpy(id, &u, sizeof(u));
+  return MS_OK;
+}
+
+extern "C" ms_status ms_nccl_comm_init(void **comm, int32_t nranks, int32_t rank, const void *id, int device) {
+  if (!comm || !id || nranks < 1 || rank < 0 || rank >= nranks || device < 0) return MS_ERR_INVALID_ARG;
+  const Nccl &N = nccl();
+  if (!N.ok) return MS_ERR_NCCL;
+  if (cudaSetDevice(device) != cudaSuccess) return MS_ERR_CUDA;
+  ncclUniqueId u;
+  memcpy(&u, id, sizeof(u));
+  ncclComm_t c = nullptr;
+  if (N.CommInitRank(&c, nranks, u, rank) != ncclSuccess) return MS_ERR_NCCL;
+  *comm = c;
+  return MS_OK;
+}
+
+extern "C" ms_status ms_nccl_comm_destroy(void *comm) {
+  if (!comm) return MS_OK;
+  const Nccl &N = nccl();
+  if (!N.ok) return MS_ERR_NCCL;
+  return N.CommDestroy((ncclComm_t)comm) == ncclSuccess ? MS_OK : MS_ERR_NCCL;
+}
+
+extern "C" ms_status ms_dist_workspace_size(ms_plan_t plan, uint64_t n_local, int32_t nranks, size_t *bytes) {
+  if (!plan || !bytes || nranks < 1) return MS_ERR_INVALID_ARG;
+  ms_bucket_spec spec;
+  int32_t kv = 0;
+  ms_status st = ms_plan_spec(plan, &spec, &kv);
+  if (st != MS_OK) return st;
+  DistLayout d = dist_layout(plan, spec.m, kv, n_local, nranks, &st);
+  if (st != MS_OK) return st;
+  *bytes = d.bytes;
+  return MS_OK;
+}
+
+extern "C" ms_status ms_dist_run(ms_plan_t plan, void *comm, const uint32_t *keys_in, const uint32_t *vals_in,
+                                 const void *ids, uint64_t n_local, uint32_t *keys_out, uint32_t *vals_out,
+                                 uint64_t out_capacity, uint64_t *offsets_global, uint64_t *win_start,
+                                 uint64_t *win_len, void *workspace, size_t workspace_bytes, void *stream) {
+  if (!plan || !comm) return MS_ERR_INVALID_ARG;
+  if ((vals_in == nullptr) != (vals_out == nullptr)) return MS_ERR_INVALID_ARG;
+  if (!keys_out || !workspace) return MS_ERR_INVALID_ARG;
+  ms_bucket_spec spec;
+  int32_t kv = 0;
+  ms_status st = ms_plan_spec(plan, &spec, &kv);
+  if (st != MS_OK) return st;
+  if (vals_in && !kv) return MS_ERR_UNSUPPORTED;
+  const Nccl &N = nccl();
+  if (!N.ok) return MS_ERR_NCCL;
+  ncclComm_t c = (ncclComm_t)comm;
+  int P = 0, rank = 0, dev = 0;
+  if (N.CommCount(c, &P) != ncclSuccess || N.CommUserRank(c, &rank) != ncclSuccess ||
+      N.CommCuDevice(c, &dev) != ncclSuccess)
+    return MS_ERR_NCCL;
+  const uint32_t m = spec.m;
+  DistLayout d = dist_layout(plan, m, vals_in != nullptr, n_local, P, &st);
+  if (st != MS_OK) return st;
+  if (workspace_bytes < d.bytes) return MS_ERR_WORKSPACE;
+  if (reinterpret_cast<uintptr_t>(workspace) & 15u) return MS_ERR_ALIGNMENT;
+  int prev = -1;
+  if (cudaGetDevice(&prev) != cudaSuccess) return MS_ERR_CUDA;
+  if (prev != dev && cudaSetDevice(dev) != cudaSuccess) return MS_ERR_CUDA;
+  struct Restore {
+    int prev, dev;
+    ~Restore() {
+      if (prev != dev) cudaSetDevice(prev);
+    }
+  } restore{prev, dev};
+  cudaStream_t s = (cudaStream_t)stream;
+  char *w = (char *)workspace;
+  uint32_t *lk = (uint32_t *)(w + d.off_keys), *lv = vals_in ? (uint32_t *)(w + d.off_vals) : nullptr;
+  uint32_t *loff = (uint32_t *)(w + d.off_loff);
+  uint64_t *cnt = (uint64_t *)(w + d.off_cnt), *gath = (uint64_t *)(w + d.off_gath);
+  // 1. local stable multisplit of the shard
+  st = ms_run(plan, keys_in, vals_in, ids, lk, lv, n_local, loff, workspace, d.local_ws, stream);
+  if (st != MS_OK) return st;
+  // 2. per-rank bucket counts, all-gathered (rows in rank order)
+  k_counts_from_offsets<<<1, 256, 0, s>>>(loff, cnt, m);
+  if (cudaGetLastError() != cudaSuccess) return MS_ERR_CUDA;
+  if (N.AllGather(cnt, gath, m, ncclUint64, c, s) != ncclSuccess) return MS_ERR_NCCL;
+  std::vector<uint64_t> counts((size_t)P * m);
+  if (cudaMemcpyAsync(counts.data(), gath, counts.size() * 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return MS_ERR_CUDA;
+  // 3. pieces
+  std::vector<ms_piece> send(m + P), recv((size_t)m * P + 1);
+  std::vector<uint64_t> offg(m + 1);
+  int32_t ns = 0, nr = 0;
+  uint64_t ws0 = 0, wl = 0;
+  st = ms_dist_pieces(P, rank, m, counts.data(), send.data(), (int32_t)send.size(), &ns, recv.data(),
+                      (int32_t)recv.size(), &nr, offg.data(), &ws0, &wl);
+  if (st != MS_OK) return st;
+  if (wl > out_capacity) return MS_ERR_INVALID_ARG;  // the caller's window buffers are too small
+  if (offsets_global) memcpy(offsets_global, offg.data(), offg.size() * 8);
+  if (win_start) *win_start = ws0;
+  if (win_len) *win_len = wl;
+  // 4. the exchange: local pieces by copy, the rest by one NCCL group of send/recv
+  for (int32_t i = 0; i < ns; ++i) {
+    const ms_piece &q = send[i];
+    if (q.peer != rank || q.len == 0) continue;
+    if (cudaMemcpyAsync(keys_out + q.dst_off, lk + q.src_off, q.len * 4, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+      return MS_ERR_CUDA;
+    if (lv && cudaMemcpyAsync(vals_out + q.dst_off, lv + q.src_off, q.len * 4, cudaMemcpyDeviceToDevice, s) !=
+                  cudaSuccess)
+      return MS_ERR_CUDA;
+  }
+  if (N.GroupStart() != ncclSuccess) return MS_ERR_NCCL;
+  ncclResult_t r = ncclSuccess;
+  for (int a = 0; a < (lv ? 2 : 1) && r == ncclSuccess; ++a) {
+    const uint32_t *src = a ? lv : lk;
+    uint32_t *dst = a ? vals_out : keys_out;
+    for (int32_t i = 0; i < ns && r == ncclSuccess; ++i)
+      if (send[i].peer != rank && send[i].len)
+        r = N.Send(src + send[i].src_off, send[i].len, ncclUint32, send[i].peer, c, s);
+    for (int32_t i = 0; i < nr && r == ncclSuccess; ++i)
+      if (recv[i].peer != rank && recv[i].len)
+        r = N.Recv(dst + recv[i].dst_off, recv[i].len, ncclUint32, recv[i].peer, c, s);
+  }
+  const ncclResult_t r2 = N.GroupEnd();
+  return (r == ncclSuccess && r2 == ncclSuccess) ? MS_OK : MS_ERR_NCCL;
+}

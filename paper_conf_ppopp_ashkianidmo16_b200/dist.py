@@ -233,4 +233,95 @@ def dist_multisplit_fused(keys, vals=None, spec=None, group=None):
     torch.cuda.current_stream().synchronize()
     dist.barrier(group)  # every rank's stores into my window are complete
     wl = int(wst[g + 1] - wst[g])
-    return bufs[0][:wl], (bufs[1][:wl] if kv else None), int(wst[g])
+    # the symmetric windows are reused by the next call (every rank scatters into them again):
+    # hand the caller tensors it owns
+    out_k = bufs[0][:wl].clone()
+    out_v = bufs[1][:wl].clone() if kv else None
+    dist.barrier(group)  # no rank starts its next scatter into my window before my copy is taken
+    return out_k, out_v, int(wst[g])
+
+
+# ---------------------------------------------------------------------------
+# ms_dist_run (include/ms.h): the whole sharded multisplit as one native collective call over an
+# NCCL communicator that libms bootstraps itself (the 128-byte unique id is broadcast over the torch
+# process group).  The count all-gather, the count differencing, the piece planning and the grouped
+# NCCL send/recv all run inside libms.so.
+class NcclComm:
+    """An ncclComm_t for ms_dist_run, one per rank of `group` (collective constructor)."""
+
+    def __init__(self, group=None, device=None):
+        import torch
+        import torch.distributed as dist
+        self.rank = dist.get_rank(group)
+        self.nranks = dist.get_world_size(group)
+        self.device = torch.cuda.current_device() if device is None else int(device)
+        uid = ctypes.create_string_buffer(128)
+        if self.rank == 0:
+            check(_abi.lib().ms_nccl_get_unique_id(uid), "ms_nccl_get_unique_id")
+        box = [bytes(uid.raw) if self.rank == 0 else None]
+        src = dist.get_global_rank(group, 0) if group is not None else 0
+        dist.broadcast_object_list(box, src=src, group=group)
+        uid = ctypes.create_string_buffer(box[0], 128)
+        self._h = ctypes.c_void_p()
+        check(_abi.lib().ms_nccl_comm_init(ctypes.byref(self._h), self.nranks, self.rank, uid, self.device),
+              "ms_nccl_comm_init")
+
+    @classmethod
+    def single(cls, device=None):
+        """A one-rank communicator (no process group needed): ms_dist_run then equals ms_run."""
+        import torch
+        self = cls.__new__(cls)
+        self.rank, self.nranks = 0, 1
+        self.device = torch.cuda.current_device() if device is None else int(device)
+        uid = ctypes.create_string_buffer(128)
+        check(_abi.lib().ms_nccl_get_unique_id(uid), "ms_nccl_get_unique_id")
+        self._h = ctypes.c_void_p()
+        check(_abi.lib().ms_nccl_comm_init(ctypes.byref(self._h), 1, 0, uid, self.device), "ms_nccl_comm_init")
+        return self
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _abi.lib().ms_nccl_comm_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class DistPlan:
+    """A plan + workspace + window buffers for repeated ms_dist_run calls on shards of up to
+    max_local elements and a global total of up to max_total elements."""
+
+    def __init__(self, spec, comm: NcclComm, max_local: int, max_total: int, with_values: bool = False):
+        import torch
+        from .api import Plan
+        self.spec, self.comm = spec, comm
+        self.plan = Plan(spec, max(int(max_local), 1), with_values=with_values, device=comm.device)
+        b = ctypes.c_size_t()
+        check(_abi.lib().ms_dist_workspace_size(self.plan._h, max(int(max_local), 1), comm.nranks, ctypes.byref(b)),
+              "ms_dist_workspace_size")
+        dev = torch.device("cuda", comm.device)
+        self.ws = torch.empty(max(b.value, 256), dtype=torch.uint8, device=dev)
+        self.cap = -(-int(max_total) // comm.nranks) + 1
+        self.out_k = torch.empty(self.cap, dtype=torch.int32, device=dev)
+        self.out_v = torch.empty(self.cap, dtype=torch.int32, device=dev) if with_values else None
+
+    def run(self, keys, vals=None, ids=None, stream=None, copy_out=True):
+        """Collective.  Returns (keys_window, vals_window, offsets_global u64[m+1] numpy, window_start).
+        copy_out=False returns views of the reused window buffers (valid until the next run)."""
+        from .api import _ptr, _stream
+        offg = np.zeros(self.spec.m + 1, dtype=np.uint64)
+        ws0, wl = ctypes.c_uint64(), ctypes.c_uint64()
+        check(_abi.lib().ms_dist_run(self.plan._h, self.comm._h, _ptr(keys), _ptr(vals), _ptr(ids), keys.numel(),
+                                     _ptr(self.out_k), _ptr(self.out_v if vals is not None else None), self.cap,
+                                     offg.ctypes.data_as(ctypes.c_void_p), ctypes.byref(ws0), ctypes.byref(wl),
+                                     _ptr(self.ws), self.ws.numel(), _stream(stream)), "ms_dist_run")
+        k = self.out_k[:wl.value]
+        v = self.out_v[:wl.value] if vals is not None else None
+        if copy_out:
+            k = k.clone()
+            v = v.clone() if v is not None else None
+        return k, v, offg, ws0.value

@@ -198,3 +198,32 @@ def test_product_path_has_no_oracle_or_fallback():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src and "liboracle" not in src, f
+
+
+def test_dist_run_argument_errors_without_gpu():
+    """ms_dist_run / the NCCL bootstrap refuse bad arguments before touching NCCL or CUDA."""
+    L = _abi.lib()
+    st, h = _create(BucketSpec("delta", 8, delta=5), max_n=4096)
+    P = ctypes.c_void_p
+    A, B, W = P(0x10000000), P(0x20000000), P(0x30000000)
+    assert L.ms_dist_run(h, None, A, None, None, 100, B, None, 100, None, None, None, W, 1 << 20, None) == \
+        _abi.MS_ERR_INVALID_ARG                                                   # no communicator
+    assert L.ms_dist_run(h, P(0x40000000), A, A, None, 100, B, None, 100, None, None, None, W, 1 << 20, None) == \
+        _abi.MS_ERR_INVALID_ARG                                                   # unpaired values
+    assert L.ms_dist_run(h, P(0x40000000), A, A, None, 100, B, B, 100, None, None, None, W, 1 << 20, None) == \
+        _abi.MS_ERR_UNSUPPORTED                                                   # values on a key-only plan
+    b = ctypes.c_size_t()
+    assert L.ms_dist_workspace_size(h, 4096, 4, ctypes.byref(b)) == _abi.MS_OK
+    ws = ctypes.c_size_t()
+    assert L.ms_plan_workspace_size(h, 4096, ctypes.byref(ws)) == _abi.MS_OK
+    assert b.value >= ws.value + 4096 * 4 + 4 * 8 * 8                             # staging + counts
+    assert L.ms_dist_workspace_size(h, 4096, 0, ctypes.byref(b)) == _abi.MS_ERR_INVALID_ARG
+    cm = ctypes.c_void_p()
+    assert L.ms_nccl_comm_init(ctypes.byref(cm), 2, 2, A, 0) == _abi.MS_ERR_INVALID_ARG   # rank >= nranks
+    assert L.ms_nccl_comm_init(None, 2, 0, A, 0) == _abi.MS_ERR_INVALID_ARG
+    assert L.ms_nccl_get_unique_id(None) == _abi.MS_ERR_INVALID_ARG
+    spec = _abi.ms_bucket_spec()
+    kv = ctypes.c_int32()
+    assert L.ms_plan_spec(h, ctypes.byref(spec), ctypes.byref(kv)) == _abi.MS_OK
+    assert spec.m == 8 and spec.delta == 5 and kv.value == 0
+    L.ms_plan_destroy(h)

@@ -171,3 +171,88 @@ def _worker(rank, P, port, n, kind, m, dist_name, mode, kv):
 def test_dist_multisplit_gloo(P, kind, m, dist_name, mode, kv):
     n = 20011
     mp.spawn(_worker, args=(P, _free_port(), n, kind, m, dist_name, mode, kv), nprocs=P, join=True)
+
+
+# ------------------------------------------------------------ the CUDA local step (GPU box)
+def _worker_cuda(rank, P, port, n, kind, m, dist_name, mode, kv):
+    """Like _worker, but every rank's local step is the product path: ms_run on cuda:0 (all ranks
+    share the one GPU of the test box), the exchange over gloo on host copies of its output."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=P)
+    try:
+        from paper_conf_ppopp_ashkianidmo16_b200.api import Plan
+        torch.cuda.set_device(0)
+        spec, ospec, ranges = _case(kind, m)
+        sizes = _shard_sizes(P, n, mode)
+        start = sum(sizes[:rank])
+        keys = W.keys_np(sizes[rank], 11, dist_name, m, ranges, start=start) if dist_name != "uniform" else \
+            W.keys_np(sizes[rank], 11, start=start)
+        vals = W.values_np(sizes[rank], 11, "index", start=start) if kv else None
+        plan = Plan(spec, max(1, sizes[rank]), with_values=kv)
+
+        def local(k, v):  # the CUDA multisplit of this rank's shard; outputs staged to the host for gloo
+            ko, vo, off = plan.run(k.cuda(), None if v is None else v.cuda())
+            torch.cuda.synchronize()
+            assert plan.last_launches() == (1 if k.numel() else 0)  # ONE at these sizes (m <= 32)
+            return ko.cpu(), (vo.cpu() if vo is not None else None), off.cpu().to(torch.int64) & 0xFFFFFFFF
+
+        kt = torch.from_numpy(keys.view(np.int32).copy())
+        vt = torch.from_numpy(vals.view(np.int32).copy()) if kv else None
+        wk, wv, offg, ws = dist_multisplit(kt, vt, spec, local=local)
+        allk = W.keys_np(n, 11, dist_name, m, ranges) if dist_name != "uniform" else W.keys_np(n, 11)
+        allv = W.values_np(n, 11, "index") if kv else None
+        eko, evo, eoff = oracle.multisplit(ospec, allk, allv)
+        assert np.array_equal(offg, eoff)
+        assert np.array_equal(wk.numpy().view(np.uint32), eko[ws:ws + wk.numel()])
+        if kv:
+            assert np.array_equal(wv.numpy().view(np.uint32), evo[ws:ws + wv.numel()])
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("P,kind,m,dist_name,mode,kv", [
+    (2, "delta", 8, "uniform", "equal", True),
+    (3, "splitters", 32, "hot", "empty", False),
+])
+def test_dist_multisplit_gloo_cuda_local(P, kind, m, dist_name, mode, kv):
+    """World size 2-3 on gloo with the REAL local step (libms ms_run on cuda:0) on every rank."""
+    n = 3 * 4096 * 148 + 1234  # several tiles per resident CTA, ragged
+    ctx = mp.get_context("spawn")
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_cuda, args=(r, P, port, n, kind, m, dist_name, mode, kv)) for r in range(P)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(600)
+    assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("delta", 256, True)])
+def test_dist_run_nccl_single_rank(kind, m, kv):
+    """ms_dist_run (the native collective: local ms_run, NCCL count all-gather, piece planning, NCCL
+    group send/recv) on a one-rank NCCL communicator: the window is the whole output and must equal
+    the oracle; offsets_global equal the oracle's offsets.  (A one-GPU box cannot host P > 1 NCCL
+    ranks -- NCCL rejects two ranks on one device; the P > 1 piece planning is pinned by the CPU
+    tests above and the exchange by the gloo runs.)"""
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import DistPlan, NcclComm
+    torch.cuda.set_device(0)
+    spec, ospec, ranges = _case(kind, m)
+    n = (1 << 22) + 333
+    keys = W.keys_np(n, 5, "binomial", m, ranges)
+    vals = W.values_np(n, 5, "index") if kv else None
+    comm = NcclComm.single(0)
+    dp = DistPlan(spec, comm, n, n, with_values=kv)
+    kd = torch.from_numpy(keys.view(np.int32).copy()).cuda()
+    vd = torch.from_numpy(vals.view(np.int32).copy()).cuda() if kv else None
+    eko, evo, eoff = oracle.multisplit(ospec, keys, vals)
+    for _ in range(2):  # repeated runs on one workspace
+        wk, wv, offg, ws = dp.run(kd, vd)
+        torch.cuda.synchronize()
+        assert ws == 0 and wk.numel() == n
+        assert np.array_equal(offg, eoff)
+        assert np.array_equal(wk.cpu().numpy().view(np.uint32), eko)
+        if kv:
+            assert np.array_equal(wv.cpu().numpy().view(np.uint32), evo)
+    comm.close()
