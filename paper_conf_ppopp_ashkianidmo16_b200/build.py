@@ -14,7 +14,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 OBJ = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libms.so")
-SOURCES = ["ms_api.cu", "ms_dist.cu", "k3_lowbits.cu", "k3_shiftc.cu", "k3_shift.cu", "k3_delta.cu", "k3_splitters.cu",
+SOURCES = ["ms_api.cu", "ms_dist.cu", "ms_wide.cu", "k3_lowbits.cu", "k3_shiftc.cu", "k3_shift.cu", "k3_delta.cu",
+           "k3_splitters.cu", "k3_shiftc_lo.cu", "k3_delta_lo.cu",
            "k3_ids.cu"]
 HEADERS = ["ms_k3_v2.cuh", "ms_kernels.cuh", "ms_device.cuh", "ms_k3_warp.cuh", "ms_k3p_args.h", "ms_ranged.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -38,6 +38,13 @@ struct ms_plan_s {
   int direct = 0;       // MS_ABLATION_DIRECT: K3 stores keys straight to global, no local reorder
   uint32_t k1s_per_sm = 8;  // splitter K1: persistent CTAs per SM (each builds the bin table once)
   int32_t last_launches;
+  // m > 256 ("wide"): two stable passes, by the low then the high digit of the id;
+  // wa / wb are the passes' plans (wb null when the high digit is always 0), wkind / wbp the full
+  // id's bucket function for the offsets pass over the sorted output
+  int wide = 0;  // 0 no, 1 computed ids (recomputed from the keys in each pass), 2 MS_IDS (u32 ids)
+  ms_plan_s *wa = nullptr, *wb = nullptr;
+  int wkind = 0;
+  BucketParams wbp;
   // per-stage trace (ms_plan_trace): one set of 4 events per traced run
   int tracing = 0;     // 0 off, 1 per-stage events, 2 whole-run events only
   int trace_mode = 1;  // mode of the recorded runs (kept after tracing stops)
@@ -181,6 +188,8 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
     case LOWBITS: return launch_k1<LOWBITS>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case SHIFTC: return launch_k1<SHIFTC>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case SHIFT: return launch_k1<SHIFT>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case SHIFTC_LO: return launch_k1<SHIFTC_LO>(p, g, keys, ids, n, H, zp, zw, flag, s);
+    case DELTA_LO: return launch_k1<DELTA_LO>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case DELTA: return launch_k1<DELTA>(p, g, keys, ids, n, H, zp, zw, flag, s);
     case SPLITTERS: return launch_k1<SPLITTERS>(p, g, keys, ids, n, H, zp, zw, flag, s);
     default: return launch_k1<IDS>(p, g, keys, ids, n, H, zp, zw, flag, s);
@@ -205,6 +214,8 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
       case LOWBITS: return k3v_launch_lowbits(a);
       case SHIFTC: return k3v_launch_shiftc(a);
       case SHIFT: return k3v_launch_shift(a);
+      case SHIFTC_LO: return k3v_launch_shiftc_lo(a);
+      case DELTA_LO: return k3v_launch_delta_lo(a);
       case DELTA: return k3v_launch_delta(a);
       case SPLITTERS: return k3v_launch_splitters(a);
       default: return k3v_launch_ids(a);
@@ -214,6 +225,8 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
     case LOWBITS: return k3w_launch_lowbits(a);
     case SHIFTC: return k3w_launch_shiftc(a);
     case SHIFT: return k3w_launch_shift(a);
+    case SHIFTC_LO: return k3w_launch_shiftc_lo(a);
+    case DELTA_LO: return k3w_launch_delta_lo(a);
     case DELTA: return k3w_launch_delta(a);
     case SPLITTERS: return k3w_launch_splitters(a);
     default: return k3w_launch_ids(a);
@@ -242,6 +255,8 @@ cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, cons
     case LOWBITS: return launch_k1r<LOWBITS>(p, g, C, keys, ids, n, HC, flag, s);
     case SHIFTC: return launch_k1r<SHIFTC>(p, g, C, keys, ids, n, HC, flag, s);
     case SHIFT: return launch_k1r<SHIFT>(p, g, C, keys, ids, n, HC, flag, s);
+    case SHIFTC_LO: return launch_k1r<SHIFTC_LO>(p, g, C, keys, ids, n, HC, flag, s);
+    case DELTA_LO: return launch_k1r<DELTA_LO>(p, g, C, keys, ids, n, HC, flag, s);
     case DELTA: return launch_k1r<DELTA>(p, g, C, keys, ids, n, HC, flag, s);
     case SPLITTERS: return launch_k1r<SPLITTERS>(p, g, C, keys, ids, n, HC, flag, s);
     default: return launch_k1r<IDS>(p, g, C, keys, ids, n, HC, flag, s);
@@ -264,6 +279,7 @@ int choose_variant(const ms_plan_s *p, uint64_t L, bool kv) {
 
 ms_status check_ws(const ms_plan_s *p, uint64_t n, void *ws, size_t ws_bytes, Geometry *g) {
   *g = geometry(p, n);
+  if (p->wide) return MS_ERR_UNSUPPORTED;  // the stage-wise calls: plans of m <= 256 only
   if (!ws || ws_bytes < g->bytes) return MS_ERR_WORKSPACE;
   if (misaligned(ws)) return MS_ERR_ALIGNMENT;
   return MS_OK;
@@ -275,6 +291,229 @@ ms_status check_common(const ms_plan_s *p, const uint32_t *keys_in, const void *
   if (n > 0 && !keys_in) return MS_ERR_INVALID_ARG;
   if (n > 0 && p->spec.kind == MS_IDS && !ids) return MS_ERR_INVALID_ARG;
   if (misaligned(keys_in) || misaligned(ids)) return MS_ERR_ALIGNMENT;
+  return MS_OK;
+}
+
+}  // namespace
+
+extern "C" ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n, int with_values,
+                                    uint32_t flags, int device);
+extern "C" ms_status ms_plan_destroy(ms_plan_t plan);
+
+namespace {
+
+constexpr uint32_t kMaxWideM = 65536;
+
+// m in (256, 65536]: a plan of two passes.  The id has e <= 16 significant bits;
+// pass A splits by its low bA = ceil(e/2) bits, pass B by the high e - bA bits (both <= 256
+// buckets, so each pass is an ordinary plan: <= 32 buckets take K3 v2, 33..256 the ballot K3).
+//   LOWBITS(s), and DELTA with delta = 2^s and m * delta >= 2^32 (id = k >> s):
+//        A = LOWBITS(s, 2^bA), B = LOWBITS(s + bA, 2^(e - bA));
+//   DELTA with delta = 2^s, m * delta < 2^32 (id = min(k >> s, m-1)):
+//        A = SHIFTC_LO (min(k >> s, m-1) & (2^bA - 1)), B = DELTA(delta * 2^bA, ((m-1) >> bA) + 1)
+//        since floor(min(q, m-1) / 2^bA) = min(floor(q / 2^bA), (m-1) >> bA);
+//   DELTA otherwise: A = DELTA_LO (the same with floor(k / delta)), B = DELTA(delta * 2^bA, ...)
+//        (floor(floor(k/delta) / 2^bA) = floor(k / (delta * 2^bA)));
+//   MS_IDS (u32 ids): the ids ride as the KEYS of two key-value passes, A = LOWBITS(0, 2^bA),
+//        B = LOWBITS(bA, 2^(e - bA)), the caller's keys (and values) as the payload.
+// B is omitted when the high digit is 0 for every key (delta * 2^bA >= 2^32).  MS_SPLITTERS
+// (more than 255 splitters) and the variant / ablation flags are not supported here.
+ms_status create_wide(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n, int with_values, uint32_t flags,
+                      int device) {
+  const uint32_t m = spec->m;
+  if (flags & ~MS_VALIDATE) return MS_ERR_UNSUPPORTED;
+  uint32_t e = ceil_log2(m), s = 0;
+  int how = 0;  // 0 bit field, 1 SHIFTC_LO, 2 DELTA_LO, 3 ids
+  switch (spec->kind) {
+    case MS_LOWBITS:
+      if (m & (m - 1)) return MS_ERR_INVALID_ARG;
+      if (spec->shift > 31 || spec->shift + e > 32) return MS_ERR_INVALID_ARG;
+      s = spec->shift;
+      break;
+    case MS_DELTA:
+      if (spec->delta < 1) return MS_ERR_INVALID_ARG;
+      if ((spec->delta & (spec->delta - 1)) == 0) {
+        s = ceil_log2(spec->delta);
+        if (((uint64_t)m << s) >= (1ull << 32)) e = 32 - s;  // id = k >> s < 2^(32-s) <= m: a bit field
+        else how = 1;
+      } else {
+        how = 2;
+      }
+      break;
+    case MS_IDS:
+      if (spec->id_bytes != 4) return spec->id_bytes == 1 ? MS_ERR_UNSUPPORTED : MS_ERR_INVALID_ARG;
+      how = 3;
+      break;
+    case MS_SPLITTERS: return MS_ERR_UNSUPPORTED;
+    default: return MS_ERR_INVALID_ARG;
+  }
+  const uint32_t bA = e > 8 ? (e + 1) / 2 : e, bB = e - bA;
+  const int kvsub = how == 3 ? 1 : with_values;
+  ms_plan_s *a = nullptr, *b = nullptr;
+  ms_bucket_spec sa{}, sb{};
+  ms_status st;
+  if (how == 0 || how == 3) {
+    sa.kind = MS_LOWBITS;
+    sa.m = 1u << bA;
+    sa.shift = s;
+    sb.kind = MS_LOWBITS;
+    sb.m = 1u << bB;
+    sb.shift = s + bA;
+  } else {
+    sa.kind = MS_DELTA;
+    sa.m = 1u << bA;
+    sa.delta = spec->delta;
+    const uint64_t db = (uint64_t)spec->delta << bA;
+    sb.kind = MS_DELTA;
+    sb.m = db < (1ull << 32) ? ((m - 1) >> bA) + 1 : 1u;
+    sb.delta = db < (1ull << 32) ? (uint32_t)db : 1u;
+  }
+  if ((st = ms_plan_create(&a, &sa, max_n, kvsub, 0, device)) != MS_OK) return st;
+  if (how == 1 || how == 2) {  // pass A: the low digit of the CLAMPED id
+    a->kkind = how == 1 ? SHIFTC_LO : DELTA_LO;
+    a->bp.shift = s;
+    a->bp.clamp = m - 1;
+    a->bp.mmask = (1u << bA) - 1;
+  }
+  if (sb.m > 1 && (st = ms_plan_create(&b, &sb, max_n, kvsub, 0, device)) != MS_OK) {
+    ms_plan_destroy(a);
+    return st;
+  }
+  ms_plan_s *p = new (std::nothrow) ms_plan_s;
+  if (!p) {
+    ms_plan_destroy(a);
+    ms_plan_destroy(b);
+    return MS_ERR_INVALID_ARG;
+  }
+  p->spec = *spec;
+  p->spec.splitters = nullptr;
+  p->max_n = max_n;
+  p->kv = with_values ? 1 : 0;
+  p->flags = flags;
+  memset(&p->bp, 0, sizeof(p->bp));
+  p->bp.m = m;
+  p->bp.mmask = m - 1;
+  p->bp.logm = e;
+  p->bp.validate = (flags & MS_VALIDATE) ? 1u : 0u;
+  p->kkind = spec->kind == MS_IDS ? IDS : spec->kind == MS_LOWBITS ? LOWBITS : DELTA;
+  p->device = a->device;
+  p->sms = a->sms;
+  p->last_launches = 0;
+  p->wide = how == 3 ? 2 : 1;
+  p->wa = a;
+  p->wb = b;
+  // the full id for the offsets pass: a bit field, min(k >> s, m-1), min(k / delta, m-1), or
+  // min(id, m-1) over the sorted ids
+  memset(&p->wbp, 0, sizeof(p->wbp));
+  p->wbp.m = m;
+  if (how == 0) {
+    p->wkind = LOWBITS;
+    p->wbp.shift = s;
+    p->wbp.mmask = e >= 32 ? 0xFFFFFFFFu : (1u << e) - 1;
+  } else if (how == 1 || how == 3) {
+    p->wkind = SHIFTC;
+    p->wbp.shift = s;
+    p->wbp.mmask = m - 1;
+  } else {
+    p->wkind = DELTA;
+    p->wbp.magic_lo = a->bp.magic_lo;
+    p->wbp.magic_hi = a->bp.magic_hi;
+    p->wbp.mmask = m - 1;
+  }
+  *plan = p;
+  return MS_OK;
+}
+
+// workspace of a wide run: [the larger pass workspace | temporaries]
+struct WideWs {
+  size_t sub, off_tk, off_tv, off_ti, off_si, bytes;
+};
+WideWs wide_ws(const ms_plan_s *p, uint64_t n) {
+  WideWs w{};
+  w.sub = geometry(p->wa, n).bytes;
+  if (p->wb) w.sub = std::max(w.sub, geometry(p->wb, n).bytes);
+  w.sub = align_up(w.sub);
+  const size_t arr = align_up(n * 4);
+  w.off_tk = w.sub;
+  w.off_tv = w.off_tk + arr;
+  w.off_ti = w.off_tv + (p->kv ? arr : 0);
+  w.off_si = w.off_ti + (p->wide == 2 ? arr : 0);
+  w.bytes = w.off_si + (p->wide == 2 ? arr : 0);
+  return w;
+}
+
+size_t plan_ws_bytes(const ms_plan_s *p, uint64_t n) { return p->wide ? wide_ws(p, n).bytes : geometry(p, n).bytes; }
+
+}  // namespace
+
+extern "C" ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, const void *ids,
+                            uint32_t *keys_out, uint32_t *vals_out, uint64_t n, uint32_t *offsets, void *ws,
+                            size_t ws_bytes, void *stream);
+
+namespace {
+
+// ms_run of a wide plan (arguments already checked by ms_run): pass A into temporaries of the
+// workspace, pass B into the outputs, then the offsets from the sorted output.
+ms_status run_wide(ms_plan_s *p, const uint32_t *keys_in, const uint32_t *vals_in, const void *ids,
+                   uint32_t *keys_out, uint32_t *vals_out, uint64_t n, uint32_t *offsets, void *ws, size_t ws_bytes,
+                   void *stream) {
+  const WideWs L = wide_ws(p, n);
+  if (!ws || ws_bytes < L.bytes) return MS_ERR_WORKSPACE;
+  if (misaligned(ws)) return MS_ERR_ALIGNMENT;
+  DeviceGuard dg(p->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  p->last_launches = 0;
+  if (n == 0) {
+    if (offsets && cudaMemsetAsync(offsets, 0, ((size_t)p->spec.m + 1) * 4, s) != cudaSuccess) return MS_ERR_CUDA;
+    return MS_OK;
+  }
+  char *w = (char *)ws;
+  uint32_t *tk = (uint32_t *)(w + L.off_tk), *tv = p->kv ? (uint32_t *)(w + L.off_tv) : nullptr;
+  uint32_t *ti = (uint32_t *)(w + L.off_ti), *si = (uint32_t *)(w + L.off_si);
+  cudaEvent_t *ev = trace_next(p);
+  if (ev) cudaEventRecord(ev[0], s);
+  int32_t launches = 0;
+  ms_status st = MS_OK;
+  auto run = [&](ms_plan_s *q, const uint32_t *k, const uint32_t *v, uint32_t *ko, uint32_t *vo) {
+    if (st != MS_OK) return;
+    st = ms_run(q, k, v, nullptr, ko, vo, n, nullptr, ws, L.sub, stream);
+    launches += q->last_launches;
+  };
+  const uint32_t *sorted;  // the id-sorted array the offsets are read from
+  if (p->wide == 1) {      // computed ids: recomputed from the keys by both passes
+    if (p->wb) {
+      run(p->wa, keys_in, vals_in, tk, tv);
+      if (ev) cudaEventRecord(ev[1], s);
+      run(p->wb, tk, tv, keys_out, vals_out);
+    } else {
+      run(p->wa, keys_in, vals_in, keys_out, vals_out);
+      if (ev) cudaEventRecord(ev[1], s);
+    }
+    sorted = keys_out;
+  } else {  // MS_IDS: the ids are the keys of both passes, the caller's keys (values) the payload
+    const uint32_t *id32 = (const uint32_t *)ids;
+    if (p->flags & MS_VALIDATE) {
+      if (cudaMemsetAsync(ws, 0, 4, s) != cudaSuccess ||
+          ids_check_launch(id32, n, p->spec.m, (uint32_t *)ws, p->sms, s) != cudaSuccess)
+        return MS_ERR_CUDA;
+      ++launches;
+    }
+    // (e >= 9 id bits for m > 256, so both digits are non-empty: wb exists)
+    run(p->wa, id32, keys_in, ti, tk);
+    if (vals_in) run(p->wa, id32, vals_in, si, tv);  // the same stable permutation (same ids)
+    if (ev) cudaEventRecord(ev[1], s);
+    run(p->wb, ti, tk, si, keys_out);
+    if (vals_in) run(p->wb, ti, tv, tk, vals_out);
+    sorted = si;
+  }
+  if (st != MS_OK) return st;
+  if (ev) cudaEventRecord(ev[2], s);
+  if (offsets) {
+    if (wide_offsets_launch(p->wkind, sorted, n, offsets, p->wbp, p->sms, s) != cudaSuccess) return MS_ERR_CUDA;
+    ++launches;
+  }
+  if (ev) cudaEventRecord(ev[3], s);
+  p->last_launches = launches;
   return MS_OK;
 }
 
@@ -303,8 +542,9 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (!plan || !spec) return MS_ERR_INVALID_ARG;
   *plan = nullptr;
   const uint32_t m = spec->m;
-  if (m < 1 || m > (uint32_t)kMaxM) return MS_ERR_INVALID_ARG;
+  if (m < 1 || m > kMaxWideM) return MS_ERR_INVALID_ARG;
   if (max_n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
+  if (m > (uint32_t)kMaxM) return create_wide(plan, spec, max_n, with_values, flags, device);
   constexpr uint32_t kVariants = MS_VARIANT_3K | MS_VARIANT_RANGED | MS_VARIANT_ONE;
   if (flags & ~(MS_VALIDATE | kVariants | MS_ABLATION_DIRECT)) return MS_ERR_INVALID_ARG;
   const uint32_t vf = flags & kVariants;
@@ -384,21 +624,31 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
 }
 
 ms_status ms_plan_destroy(ms_plan_t plan) {
-  if (plan)
+  if (plan) {
     for (cudaEvent_t e : plan->trace_ev) cudaEventDestroy(e);
+    ms_plan_destroy(plan->wa);
+    ms_plan_destroy(plan->wb);
+  }
   delete plan;
   return MS_OK;
 }
 
 ms_status ms_plan_workspace_size(ms_plan_t p, uint64_t n, size_t *bytes) {
   if (!p || !bytes || n > p->max_n) return MS_ERR_INVALID_ARG;
-  *bytes = geometry(p, n).bytes;
+  *bytes = plan_ws_bytes(p, n);
   return MS_OK;
 }
 
 ms_status ms_plan_geometry(ms_plan_t p, uint64_t n, uint32_t *tile, uint64_t *num_tiles,
                            int32_t *variant) {
   if (!p || n > p->max_n) return MS_ERR_INVALID_ARG;
+  if (p->wide) {  // the first pass's tiles; variant 3 = two passes
+    Geometry g = geometry(p->wa, n);
+    if (tile) *tile = g.T;
+    if (num_tiles) *num_tiles = g.L;
+    if (variant) *variant = 3;
+    return MS_OK;
+  }
   Geometry g = geometry(p, n);
   if (tile) *tile = g.T;
   if (num_tiles) *num_tiles = g.L;
@@ -557,6 +807,7 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
       overlap(keys_out, nb, vals_out, nb) ||
       overlap(keys_out, nb, ids, n * p->spec.id_bytes) || overlap(vals_out, nb, ids, n * p->spec.id_bytes))
     return MS_ERR_ALIAS;
+  if (p->wide) return run_wide(p, keys_in, vals_in, ids, keys_out, vals_out, n, offsets, ws, ws_bytes, stream);
   Geometry g;
   if ((st = check_ws(p, n, ws, ws_bytes, &g)) != MS_OK) return st;
   DeviceGuard dg(p->device);
@@ -641,7 +892,7 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
 
 ms_status ms_plan_workspace_size_host(ms_plan_t p, uint64_t n, size_t *bytes) {
   if (!p || !bytes || n > p->max_n) return MS_ERR_INVALID_ARG;
-  size_t ws = geometry(p, n).bytes;
+  size_t ws = plan_ws_bytes(p, n);
   size_t arr = align_up(n * 4);
   size_t stage = arr * (p->kv ? 4 : 2) + (p->spec.kind == MS_IDS ? align_up(n * p->spec.id_bytes) : 0) +
                  align_up((p->spec.m + 1) * 4);
@@ -663,8 +914,8 @@ ms_status ms_run_host(ms_plan_t p, const uint32_t *keys_h, const uint32_t *vals_
   if (misaligned(ws)) return MS_ERR_ALIGNMENT;
   DeviceGuard dg(p->device);
   cudaStream_t s = (cudaStream_t)stream;
-  Geometry g = geometry(p, n);
-  char *w = (char *)ws + g.bytes;
+  const size_t wsb = plan_ws_bytes(p, n);
+  char *w = (char *)ws + wsb;
   size_t arr = align_up(n * 4);
   uint32_t *dk = (uint32_t *)w; w += arr;
   uint32_t *dko = (uint32_t *)w; w += arr;
@@ -680,7 +931,7 @@ ms_status ms_run_host(ms_plan_t p, const uint32_t *keys_h, const uint32_t *vals_
       return MS_ERR_CUDA;
   }
   ms_status st = ms_run(p, keys_h ? dk : nullptr, vals_h ? dv : nullptr, did, dko, vals_h ? dvo : nullptr, n,
-                        offsets_h ? doff : nullptr, ws, g.bytes, stream);
+                        offsets_h ? doff : nullptr, ws, wsb, stream);
   if (st != MS_OK) return st;
   if (n > 0) {
     if (cudaMemcpyAsync(keys_out_h, dko, n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess) return MS_ERR_CUDA;

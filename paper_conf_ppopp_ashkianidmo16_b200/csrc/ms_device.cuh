@@ -12,7 +12,11 @@ namespace ms {
 // these; MS_DELTA becomes SHIFTC when delta is a power of two (incl. 1), and
 // SHIFT when in addition m * delta >= 2^32 (the clamp can never fire: the
 // paper's "buckets equally divide the 32-bit domain").
-enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3, SHIFTC = 4, SHIFT = 5 };
+// SHIFTC_LO / DELTA_LO: the LOW digit of a clamped id, (min(q, clamp) & mmask)
+// with q = k >> shift or floor(k / delta) -- the first pass of the two-pass
+// multisplit for m > 256 (ms_api.cu "wide plans").
+enum Kind : int { LOWBITS = 0, DELTA = 1, SPLITTERS = 2, IDS = 3, SHIFTC = 4, SHIFT = 5, SHIFTC_LO = 6,
+                  DELTA_LO = 7 };
 
 constexpr int kThreads = 256;  // CTA = 8 warps (the paper's NW = 8)
 constexpr int kWarps = kThreads / 32;
@@ -31,6 +35,7 @@ struct BucketParams {
   uint32_t logm;      // ceil(log2 m): splitter search steps
   uint32_t id_bytes;  // IDS: 1 or 4
   uint32_t validate;  // IDS: flag ids >= m
+  uint32_t clamp;     // SHIFTC_LO / DELTA_LO: the full id's clamp (m_full - 1)
   uint32_t spl[kMaxM];
 };
 
@@ -47,10 +52,13 @@ __device__ __forceinline__ uint32_t id_shiftc(uint32_t k, const BucketParams &p)
 // id = min(floor(k / delta), m - 1) for 1 < delta < 2^32, not a power of two:
 // floor(k * c / 2^64) with c = ceil(2^64 / delta) is exact for every 32-bit k
 // (F = 64 >= N + log2(delta) = 32 + 32).  Two 32x32->64 multiply-adds.
-__device__ __forceinline__ uint32_t id_delta(uint32_t k, const BucketParams &p) {
+__device__ __forceinline__ uint32_t div_delta(uint32_t k, const BucketParams &p) {
   const uint64_t lo = (uint64_t)p.magic_lo * k;
   const uint64_t hi = (uint64_t)p.magic_hi * k + (lo >> 32);
-  return min((uint32_t)(hi >> 32), p.mmask);
+  return (uint32_t)(hi >> 32);
+}
+__device__ __forceinline__ uint32_t id_delta(uint32_t k, const BucketParams &p) {
+  return min(div_delta(k, p), p.mmask);
 }
 
 // id = #{ j : s_j < k }: branchless binary search over the padded table.
@@ -111,6 +119,8 @@ __device__ __forceinline__ uint32_t bucket_of_key(uint32_t k, const BucketParams
   else if constexpr (KIND == SHIFT) return k >> p.shift;  // m * delta >= 2^32: always < m
   else if constexpr (KIND == SHIFTC) return id_shiftc(k, p);
   else if constexpr (KIND == DELTA) return id_delta(k, p);
+  else if constexpr (KIND == SHIFTC_LO) return min(k >> p.shift, p.clamp) & p.mmask;
+  else if constexpr (KIND == DELTA_LO) return min(div_delta(k, p), p.clamp) & p.mmask;
   else if constexpr (KIND == SPLITTERS) return id_splitters(k, spl_s, p.logm);
   else return 0u;
 }

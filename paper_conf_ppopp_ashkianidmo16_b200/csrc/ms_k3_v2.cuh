@@ -107,7 +107,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   constexpr int NCH = K / 4;  // 16-byte chunks per thread block
   constexpr int LOGNT = NT == 256 ? 8 : 7;
   // multi-instruction (and precomputed) ids are kept in registers, one byte per key, not recomputed
-  constexpr bool KEEP_ID = KIND == SPLITTERS || KIND == DELTA || KIND == IDS;
+  constexpr bool KEEP_ID = KIND == SPLITTERS || KIND == DELTA || KIND == IDS || KIND == SHIFTC_LO || KIND == DELTA_LO;
   static_assert(KIND != IDS || IDB == 1 || IDB == 4, "IDS needs IDB = 1 or 4");
   const uint32_t mm4 = p.mmask * 0x01010101u;  // IDS: per-byte clamp bound
   uint32_t bad = 0;                            // IDS: some raw id > m - 1 (validation)

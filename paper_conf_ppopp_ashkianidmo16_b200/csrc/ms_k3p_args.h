@@ -207,6 +207,8 @@ cudaError_t k3v_launch_shift(const K3pArgs &a);
 cudaError_t k3v_launch_delta(const K3pArgs &a);
 cudaError_t k3v_launch_splitters(const K3pArgs &a);
 cudaError_t k3v_launch_ids(const K3pArgs &a);
+cudaError_t k3v_launch_shiftc_lo(const K3pArgs &a);
+cudaError_t k3v_launch_delta_lo(const K3pArgs &a);
 // m > 32: warp-ballot K3 (ms_k3_warp.cuh); kpt carries the rounds per warp R (8 or 16)
 cudaError_t k3w_launch_lowbits(const K3pArgs &a);
 cudaError_t k3w_launch_shiftc(const K3pArgs &a);
@@ -214,5 +216,11 @@ cudaError_t k3w_launch_shift(const K3pArgs &a);
 cudaError_t k3w_launch_delta(const K3pArgs &a);
 cudaError_t k3w_launch_splitters(const K3pArgs &a);
 cudaError_t k3w_launch_ids(const K3pArgs &a);
+cudaError_t k3w_launch_shiftc_lo(const K3pArgs &a);
+cudaError_t k3w_launch_delta_lo(const K3pArgs &a);
+// m > 256 (ms_wide.cu): offsets from the id-sorted output, MS_IDS range check
+cudaError_t wide_offsets_launch(int kind, const uint32_t *src, uint64_t n, uint32_t *offsets,
+                                const BucketParams &bp, int sms, cudaStream_t s);
+cudaError_t ids_check_launch(const uint32_t *ids, uint64_t n, uint32_t m, uint32_t *flag, int sms, cudaStream_t s);
 
 }  // namespace ms

@@ -227,3 +227,28 @@ def test_dist_run_argument_errors_without_gpu():
     assert L.ms_plan_spec(h, ctypes.byref(spec), ctypes.byref(kv)) == _abi.MS_OK
     assert spec.m == 8 and spec.delta == 5 and kv.value == 0
     L.ms_plan_destroy(h)
+
+
+def test_wide_plans_without_gpu():
+    """m in (256, 65536] (two-pass plans): accepted kinds, rejected ones, geometry and
+    workspace (both pass temporaries)."""
+    L = _abi.lib()
+    for spec, kv in ((BucketSpec("lowbits", 65536), 0), (BucketSpec("delta", 1000, delta=4000037), 1),
+                     (BucketSpec("delta", 300, delta=1 << 20), 0), (BucketSpec("ids", 4096, id_bytes=4), 1)):
+        st, h = _create(spec, max_n=1 << 20, kv=kv)
+        assert st == _abi.MS_OK, spec.kind
+        v, b = ctypes.c_int32(), ctypes.c_size_t()
+        assert L.ms_plan_geometry(h, 1 << 20, None, None, ctypes.byref(v)) == 0 and v.value == _abi.VARIANT_WIDE
+        assert L.ms_plan_workspace_size(h, 1 << 20, ctypes.byref(b)) == 0
+        assert b.value >= (1 << 20) * 4 * (1 + kv + (2 if spec.kind == "ids" else 0))
+        P = ctypes.c_void_p
+        # the stage-wise calls are for plans of m <= 256
+        assert L.ms_prescan(h, P(0x10000000), P(0x20000000) if spec.kind == "ids" else None, 100, P(0x30000000),
+                            P(0x40000000), 1 << 30, None) == _abi.MS_ERR_UNSUPPORTED
+        L.ms_plan_destroy(h)
+    assert _create(BucketSpec("lowbits", 65537 + 65535))[0] == _abi.MS_ERR_INVALID_ARG      # m > 65536
+    assert _create(BucketSpec("delta", 65537, delta=3))[0] == _abi.MS_ERR_INVALID_ARG
+    assert _create(BucketSpec("splitters", 300, splitters=list(range(299))))[0] == _abi.MS_ERR_UNSUPPORTED
+    assert _create(BucketSpec("ids", 300, id_bytes=1))[0] == _abi.MS_ERR_UNSUPPORTED
+    assert _create(BucketSpec("delta", 1000, delta=5), flags=2)[0] == _abi.MS_ERR_UNSUPPORTED
+    assert _create(BucketSpec("lowbits", 1024, shift=23))[0] == _abi.MS_ERR_INVALID_ARG     # shift + log2 m > 32

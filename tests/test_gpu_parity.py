@@ -42,8 +42,12 @@ def _run_case(case, variant=None, want_offsets=True, expect_variant=None):
         assert v == FORCED[variant], f"geometry reports variant {v} for forced {variant}"
     if expect_variant is not None:
         assert v == expect_variant, f"variant {v}, expected {expect_variant}"
-    assert plan.last_launches() == (_abi.LAUNCHES[v] if n else 0), \
-        f"{plan.last_launches()} launches for variant {v} (n={n})"
+    if v == _abi.VARIANT_WIDE:  # m > 256: two passes (each 1..3 launches) + the offsets pass
+        assert (2 <= plan.last_launches() <= 2 * 3 * (2 if spec.kind == "ids" else 1) + 2) if n else \
+            plan.last_launches() == 0
+    else:
+        assert plan.last_launches() == (_abi.LAUNCHES[v] if n else 0), \
+            f"{plan.last_launches()} launches for variant {v} (n={n})"
     return from_dev(ko), from_dev(vo), (None if off is None else from_dev(off)), plan
 
 
@@ -405,3 +409,67 @@ def test_parity_direct_ablation(m):
             case = make_case("delta", m, n, seed=2 * (400 + i), kv=kv)  # even seed: delta = 2^32 / m
             assert case["spec_kw"]["delta"] == (1 << 32) // m
             _assert_equal(case, _run_case(case, "direct"), _expect(case), f"direct m={m} n={n} kv={kv}")
+
+
+# ---------------------------------------------------------------- m > 256
+WIDE = [("lowbits", 512, dict(shift=0)), ("lowbits", 65536, dict(shift=7)), ("lowbits", 1024, dict(shift=22)),
+        ("delta", 300, dict(delta=1 << 20)),        # power of two, m * delta < 2^32: clamped (SHIFTC_LO + B)
+        ("delta", 1000, dict(delta=1 << 22)),
+        ("delta", 4096, dict(delta=1 << 20)),       # m * delta = 2^32: a bit field (LOWBITS passes)
+        ("delta", 65536, dict(delta=1 << 16)),
+        ("delta", 777, dict(delta=5000003)),        # magic division (DELTA_LO + DELTA)
+        ("delta", 3000, dict(delta=123457)),        # far pile holds most keys
+        ("delta", 65535, dict(delta=3)),
+        ("delta", 400, dict(delta=400000000)),      # high digit always 0: one pass + offsets
+        ("ids", 257, dict(id_bytes=4)), ("ids", 5000, dict(id_bytes=4)), ("ids", 65536, dict(id_bytes=4))]
+
+
+def _wide_case(kind, m, kw, n, seed, kv, dist="uniform"):
+    ospec = oracle.Spec(kind, m, shift=kw.get("shift", 0), delta=kw.get("delta", 1), id_bytes=kw.get("id_bytes", 1))
+    ids = None
+    if kind == "ids":
+        keys = W.keys_np(n, seed)
+        ids = W.bucket_draw_np(n, seed, "buckets" if dist == "uniform" else dist, m).astype(np.uint32)
+    elif kind == "delta" and dist != "uniform":
+        keys = W.keys_np(n, seed, dist, m, W.ranges_delta(m, kw["delta"]))
+    else:
+        keys = W.keys_np(n, seed)
+    vals = W.values_np(n, seed, "index") if kv else None
+    return dict(spec_kw=dict(kind=kind, m=m, **kw), ospec=ospec, keys=keys, vals=vals, ids=ids)
+
+
+@pytest.mark.parametrize("kind,m,kw", WIDE)
+def test_parity_wide(kind, m, kw):
+    """m in (256, 65536]: two stable passes (low digit, high digit) + offsets from the sorted output,
+    bit-exact vs the oracle on ragged sizes, KO and KV, uniform and skewed."""
+    for i, n in enumerate([0, 1, 31, 4095, 100003, (1 << 20) + 7]):
+        for kv in (False, True):
+            for dist in (["uniform", "binomial", "hot"] if (kind != "lowbits" and n > 4095) else ["uniform"]):
+                case = _wide_case(kind, m, kw, n, seed=31 * m + i, kv=kv, dist=dist)
+                got = _run_case(case)
+                _assert_equal(case, got, _expect(case), f"wide {kind} m={m} {kw} n={n} kv={kv} {dist}")
+                assert got[3].geometry(max(n, 1))[2] == 3
+
+
+@pytest.mark.parametrize("kind,m,kw,n,kv", [("delta", 65536, dict(delta=1 << 16), 1 << 28, False),
+                                            ("delta", 4096, dict(delta=1 << 20), (1 << 26) + 3, True),
+                                            ("delta", 1000, dict(delta=4000037), 1 << 26, False),
+                                            ("ids", 4096, dict(id_bytes=4), (1 << 25) + 1, True)])
+def test_parity_wide_large(kind, m, kw, n, kv):
+    """m > 256 at up to 2^28 keys, full compare (the Fig. 4-style sweep's sizes)."""
+    case = _wide_case(kind, m, kw, n, seed=4242, kv=kv)
+    _assert_equal(case, _run_case(case), _expect(case), f"wide {kind} m={m} n={n}")
+
+
+def test_wide_validate_flags_out_of_range_ids():
+    P = _pkg()
+    n, m = 100000, 1000
+    ids = W.bucket_draw_np(n, 3, "buckets", m).astype(np.uint32)
+    keys = W.keys_np(n, 3)
+    plan = P.Plan(P.BucketSpec.precomputed(m, 4), n, validate=True)
+    plan.run(to_dev(keys), ids=to_dev(ids))
+    assert plan.check() == 0
+    bad = ids.copy()
+    bad[12345] = 1000
+    plan.run(to_dev(keys), ids=to_dev(bad))
+    assert plan.check() == -8

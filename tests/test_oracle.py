@@ -182,7 +182,8 @@ def test_out_of_range_id_rejected():
 
 
 # ---------------------------------------------------------------- invariants
-@pytest.mark.parametrize("kind,m", [("delta", 8), ("splitters", 32), ("lowbits", 256), ("delta", 256)])
+@pytest.mark.parametrize("kind,m", [("delta", 8), ("splitters", 32), ("lowbits", 256), ("delta", 256),
+                                    ("delta", 1000), ("lowbits", 4096), ("splitters", 700)])
 def test_invariants_large(kind, m):
     """Permutation, id order, stability, offsets (BJ north_star invariants) at n = 2^16 + 5."""
     import workloads
@@ -208,7 +209,7 @@ def test_invariants_large(kind, m):
 def test_identity_buckets_is_stable_sort():
     """Identity buckets B_i = {i}: multisplit == stable sort of keys in [0, m)."""
     rng = np.random.default_rng(3)
-    for m in [2, 7, 32, 256]:
+    for m in [2, 7, 32, 256, 257, 4096, 65536]:   # m > 256: SURVEY NEXT-3 (P:1888-1954)
         keys = rng.integers(0, m, size=5000).astype(np.uint32)
         vals = np.arange(5000, dtype=np.uint32)
         ko, vo, _ = oracle.multisplit(oracle.Spec("delta", m, delta=1), keys, vals)
