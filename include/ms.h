@@ -102,12 +102,19 @@ typedef struct ms_plan_s *ms_plan_t;
  * MS_ABLATION_DIRECT: the paper's "Direct" post-scan (Table 4):
  * no local reorder, every key stored straight to its global position (tile
  * variant; implemented for MS_DELTA with m <= 32 and m * delta = 2^32 only,
- * else MS_ERR_UNSUPPORTED) -- a design-space ablation, same result. */
+ * else MS_ERR_UNSUPPORTED) -- a design-space ablation, same result.
+ * MS_ABLATION_NW2 / MS_ABLATION_NW4: the post-scan CTA has 2 / 4 warps instead
+ * of 8 (tile T = 1024 / 2048 keys; the local reorder then spans fewer warps,
+ * the B200 analogue of the paper's NW sweep and of warp- vs block-level
+ * reordering); ranged variant, same kinds as
+ * MS_ABLATION_DIRECT.  At most one MS_ABLATION_* flag, none with MS_VARIANT_*. */
 #define MS_VALIDATE        1u  /* flag precomputed ids >= m on the device; ms_plan_check reports it */
 #define MS_VARIANT_3K      2u
 #define MS_VARIANT_RANGED  4u
 #define MS_VARIANT_ONE     8u
 #define MS_ABLATION_DIRECT 16u
+#define MS_ABLATION_NW2    32u
+#define MS_ABLATION_NW4    64u
 
 /* Create a plan for up to max_n elements (max_n < 2^32) on CUDA device
  * `device` (-1: the calling thread's current device; every later call of the

@@ -80,7 +80,8 @@ def _check_tensor(t, name):
 
 
 VARIANT_FLAGS = {None: 0, "3k": _abi.MS_VARIANT_3K, "tile": _abi.MS_VARIANT_3K, "ranged": _abi.MS_VARIANT_RANGED,
-                 "one": _abi.MS_VARIANT_ONE, "direct": _abi.MS_ABLATION_DIRECT}
+                 "one": _abi.MS_VARIANT_ONE, "direct": _abi.MS_ABLATION_DIRECT, "nw2": _abi.MS_ABLATION_NW2,
+                 "nw4": _abi.MS_ABLATION_NW4}
 
 
 class Plan:

@@ -552,10 +552,12 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (max_n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
   if (m > (uint32_t)kMaxM) return create_wide(plan, spec, max_n, with_values, flags, device);
   constexpr uint32_t kVariants = MS_VARIANT_3K | MS_VARIANT_RANGED | MS_VARIANT_ONE;
-  if (flags & ~(MS_VALIDATE | kVariants | MS_ABLATION_DIRECT)) return MS_ERR_INVALID_ARG;
-  const uint32_t vf = flags & kVariants;
+  constexpr uint32_t kAblations = MS_ABLATION_DIRECT | MS_ABLATION_NW2 | MS_ABLATION_NW4;
+  if (flags & ~(MS_VALIDATE | kVariants | kAblations)) return MS_ERR_INVALID_ARG;
+  const uint32_t vf = flags & kVariants, af = flags & kAblations;
   if (vf & (vf - 1)) return MS_ERR_INVALID_ARG;  // at most one variant flag
-  if ((flags & MS_ABLATION_DIRECT) && vf) return MS_ERR_INVALID_ARG;
+  if (af & (af - 1)) return MS_ERR_INVALID_ARG;  // at most one ablation
+  if (af && vf) return MS_ERR_INVALID_ARG;
   if ((flags & MS_VARIANT_ONE) && m > 32) return MS_ERR_UNSUPPORTED;
   BucketParams bp;
   memset(&bp, 0, sizeof(bp));
@@ -598,8 +600,8 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
       break;
     default: return MS_ERR_INVALID_ARG;
   }
-  // the Direct ablation is instantiated for one bucket kind only (DELTA with m * delta = 2^32)
-  if ((flags & MS_ABLATION_DIRECT) && (m > 32 || kkind != SHIFT)) return MS_ERR_UNSUPPORTED;
+  // the ablations are instantiated for one bucket kind only (DELTA with m * delta = 2^32)
+  if (af && (m > 32 || kkind != SHIFT)) return MS_ERR_UNSUPPORTED;
   if (device < -1) return MS_ERR_INVALID_ARG;
   if (device == -1 && cudaGetDevice(&device) != cudaSuccess) {
     cudaGetLastError();
@@ -625,6 +627,10 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->forced = (flags & MS_VARIANT_3K) ? V_TILE : (flags & MS_VARIANT_RANGED) ? V_RANGED
             : (flags & MS_VARIANT_ONE) ? V_ONE : -1;
   p->direct = (flags & MS_ABLATION_DIRECT) ? 1 : 0;
+  if (flags & (MS_ABLATION_NW2 | MS_ABLATION_NW4)) {  // 2 / 4 warps per K3 CTA: T = 1024 / 2048, ranged
+    p->k3nt = (flags & MS_ABLATION_NW2) ? 64u : 128u;
+    p->forced = V_RANGED;
+  }
   *plan = p;
   return MS_OK;
 }

@@ -105,7 +105,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   constexpr int MP = Ly::MP, K = Ly::K, T = Ly::T, TB = Ly::TB, RS = Ly::RS;
   constexpr int NW = NT / 32;
   constexpr int NCH = K / 4;  // 16-byte chunks per thread block
-  constexpr int LOGNT = NT == 256 ? 8 : 7;
+  constexpr int LOGNT = NT == 256 ? 8 : NT == 128 ? 7 : 6;
+  static_assert(NT == 64 || NT == 128 || NT == 256, "NT");
   // multi-instruction (and precomputed) ids are kept in registers, one byte per key, not recomputed
   constexpr bool KEEP_ID = KIND == SPLITTERS || KIND == DELTA || KIND == IDS || KIND == SHIFTC_LO || KIND == DELTA_LO;
   static_assert(KIND != IDS || IDB == 1 || IDB == 4, "IDS needs IDB = 1 or 4");
@@ -672,6 +673,22 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
             else bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
             bulk_commit();
           }
+        } else if constexpr (SPB == 2) {  // (NT = 64) sub 0: head, tail, keys body; sub 1: values body
+          if (sub == 0) {
+            for (uint32_t i = 0; i < head; ++i) {
+              keys_out[Gd + i] = keys_s[P + i];
+              if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+            }
+            for (uint32_t i = head + body; i < len; ++i) {
+              keys_out[Gd + i] = keys_s[P + i];
+              if constexpr (KV) vals_out[Gd + i] = vals_s[P + i];
+            }
+          }
+          if (body && (sub == 0 || KV)) {
+            if (sub == 0) bulk_s2g(keys_out + Gd + head, keys_s + P + head, body * 4u);
+            else bulk_s2g(vals_out + Gd + head, vals_s + P + head, body * 4u);
+            bulk_commit();
+          }
         } else {  // SPB == 4: head / tail / keys body / values body
           if (sub < 2) {
             const uint32_t i0 = sub == 0 ? 0u : head + body, i1 = sub == 0 ? head : len;
@@ -737,7 +754,7 @@ template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ON
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   constexpr int KPT = 16;
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
-  constexpr int MINB = KV ? 2 : 3;
+  constexpr int MINB = (KV ? 2 : 3) * (256 / NT);
   auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE, DIRECT, IDB>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -767,6 +784,14 @@ template <int KIND, bool KV, int LOGMP, int IDB>
 inline cudaError_t k3v_launch_n(const K3pArgs &a) {
   constexpr int NT = 256;
   constexpr int STAGES = KV ? 1 : (LOGMP <= 3 ? 3 : 2);  // m <= 8 key-only: 3 stages still fit 3 CTAs/SM
+  if (a.nt != 256) {  // ablation (NW sweep): 2 or 4 warps per CTA, ranged variant, one bucket kind
+    if constexpr (KIND == SHIFT) {
+      if (a.ranged != 1) return cudaErrorNotSupported;
+      return a.nt == 128 ? k3v_launch_one<KIND, KV, LOGMP, 128, STAGES, true>(a)
+                         : k3v_launch_one<KIND, KV, LOGMP, 64, STAGES, true>(a);
+    }
+    return cudaErrorNotSupported;
+  }
   if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true, false, IDB>(a);
   if (a.direct) {  // ablation: instantiated for the one-shift bucket kind only (SHIFT: DELTA with m*delta = 2^32)
     if constexpr (KIND == SHIFT) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, true>(a);

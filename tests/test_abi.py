@@ -47,7 +47,8 @@ def _create(spec: BucketSpec, max_n=1 << 20, kv=0, flags=0, device=-1):
     (BucketSpec("delta", 8, delta=5), 4 | 8),
     (BucketSpec("delta", 8, delta=5), 2 | 8),
     (BucketSpec("delta", 8, delta=1 << 29), 16 | 2),  # ablation + forced variant
-    (BucketSpec("delta", 8, delta=5), 64),         # unknown flag
+    (BucketSpec("delta", 8, delta=5), 128),        # unknown flag
+    (BucketSpec("delta", 8, delta=1 << 29), 32 | 64),  # two ablations
 ])
 def test_plan_create_rejects(spec, flags):
     st, h = _create(spec, flags=flags)
@@ -74,6 +75,8 @@ def test_plan_create_accepts(spec):
     (BucketSpec("delta", 8, delta=5), 16),         # Direct ablation: DELTA with m * delta = 2^32 only
     (BucketSpec("delta", 64, delta=1 << 26), 16),
     (BucketSpec("ids", 8), 16),
+    (BucketSpec("delta", 8, delta=5), 32),         # NW ablations: the same one bucket kind
+    (BucketSpec("delta", 64, delta=1 << 26), 64),
 ])
 def test_plan_create_unsupported(spec, flags):
     st, h = _create(spec, flags=flags)

@@ -21,7 +21,7 @@ def _pkg():
     return P
 
 
-FORCED = {"3k": 0, "tile": 0, "direct": 0, "ranged": 1, "one": 2}
+FORCED = {"3k": 0, "tile": 0, "direct": 0, "ranged": 1, "one": 2, "nw2": 1, "nw4": 1}
 
 
 def _run_case(case, variant=None, want_offsets=True, expect_variant=None):
@@ -489,3 +489,20 @@ def test_parity_ranged_wide_m(kind, m, kv):
     n = 8 * sms * T + 5
     case = make_case(kind, m, n, seed=77, kv=kv)
     _assert_equal(case, _run_case(case, expect_variant=1), _expect(case), f"default ranged {kind} m={m}")
+
+
+@pytest.mark.parametrize("variant", ["nw2", "nw4"])
+@pytest.mark.parametrize("m", [2, 4, 8, 16, 32])
+def test_parity_nw_ablation(variant, m):
+    """The NW sweep ablation (MS_ABLATION_NW2 / NW4: 2 or 4 warps per post-scan CTA, T = 1024 / 2048,
+    the local reorder spanning fewer warps; ranged variant, 2 launches), bit-exact on ragged sizes
+    around the range boundaries, KO and KV."""
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    T = 1024 if variant == "nw2" else 2048
+    for i, n in enumerate([1, T - 1, T + 1, 100003, 37 * sms * T + 11, (1 << 22) + 3]):
+        for kv in (False, True):
+            case = make_case("delta", m, n, seed=2 * (600 + i), kv=kv, dist="binomial" if i % 2 else "uniform")
+            assert case["spec_kw"]["delta"] == (1 << 32) // m  # even seed: the SHIFT kind
+            got = _run_case(case, variant)
+            assert got[3].geometry(n)[0] == T
+            _assert_equal(case, got, _expect(case), f"{variant} m={m} n={n} kv={kv}")

@@ -1,11 +1,19 @@
-"""Design-space ablation (the paper's Table 4 question on B200): does the local
-reorder pay?  For m in {2,4,8,16,32}, key-only and key-value, DELTA buckets that equally divide the
-32-bit domain (one shift), n = 2^25 and 2^28, time (G keys/s, L2 flushed, CUDA events):
-  reorder  -- the default path (ONE launch for key-only, ranged/tile otherwise)
-  tile     -- the 3-kernel tile variant with the local reorder (plan flag MS_VARIANT_3K)
-  direct   -- the 3-kernel tile variant WITHOUT the local reorder: every key stored from registers
-              straight to its global position (MS_ABLATION_DIRECT; the paper's "Direct" method)
-Writes a markdown table to stdout.  usage: python tools/ablation.py [steps]"""
+"""Design-space ablation on B200 (the paper's Table 4 / Table 6 / §6.1 questions).
+
+Table 4 analogue: per-stage time (pre-scan / scan / post-scan, ms) and G keys/s of
+every post-scan method for m in {2, 8, 32}, key-only and key-value, n = 2^25, DELTA buckets that
+equally divide the 32-bit domain (one shift), L2 flushed, CUDA events:
+  direct  -- tile variant WITHOUT the local reorder: every key stored from registers straight to
+             its global position (MS_ABLATION_DIRECT; the paper's "Direct" method)
+  nw2     -- local reorder over 2 warps (1024-key tiles; MS_ABLATION_NW2, ranged variant): the
+             B200 analogue of the paper's warp-level reordering
+  nw4     -- reorder over 4 warps (2048-key tiles; MS_ABLATION_NW4, ranged)
+  tile    -- block-level reorder over 8 warps (4096-key tiles), K1 -> K2 -> K3 (MS_VARIANT_3K)
+  ranged  -- the same over CTA ranges, K1r -> K3 (MS_VARIANT_RANGED)
+  one     -- the same in one cooperative launch (MS_VARIANT_ONE)
+nw2 / nw4 / ranged together are the NW (warps per CTA) sweep of §6.1.
+Per-stage times come from the per-stage trace (no PDL between kernels); G keys/s from the
+whole-run trace.  usage: python tools/ablation.py [steps] [log2 n] > profiles/r02_ablation.md"""
 import os
 import sys
 
@@ -16,16 +24,18 @@ import bench  # noqa: E402
 import workloads as W  # noqa: E402
 
 steps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
-modes = {"reorder": None, "tile": "3k", "direct": "direct"}
-print("| n | mode | m | KO G keys/s | KO K3 ms | KV G keys/s | KV K3 ms |")
-print("|---|---|---|---|---|---|---|")
-for e in (25, 28):
-    for m in (2, 4, 8, 16, 32):
-        for mode, variant in modes.items():
-            row = []
-            for kv in (False, True):
-                cfg = dict(desc=f"delta m={m}", kind="delta", m=m, delta=(1 << 32) // m, n=1 << e, kv=kv,
-                           dist="uniform", seed=W.SEEDS["C4"], variant=variant)
-                r = bench.bench_config(f"abl_{m}", cfg, steps, 3, torch.device("cuda"), 1, 0, with_e2e=False)
-                row += [f"{r['value']:.1f}", f"{r['stages_ms']['k3_postscan']:.4f}"]
-            print(f"| 2^{e} | {mode} | {m} | " + " | ".join(row) + " |", flush=True)
+e = int(sys.argv[2]) if len(sys.argv) > 2 else 25
+modes = ["direct", "nw2", "nw4", "tile", "ranged", "one"]
+variant = {"direct": "direct", "nw2": "nw2", "nw4": "nw4", "tile": "3k", "ranged": "ranged", "one": "one"}
+print(f"| m | mode | method | launches | pre-scan ms | scan ms | post-scan ms | total ms (traced) | G keys/s |")
+print("|---|---|---|---|---|---|---|---|---|")
+for m in (2, 8, 32):
+    for kv in (False, True):
+        for mode in modes:
+            cfg = dict(desc=f"delta m={m}", kind="delta", m=m, delta=(1 << 32) // m, n=1 << e, kv=kv,
+                       dist="uniform", seed=W.SEEDS["C4"], variant=variant[mode])
+            r = bench.bench_config(f"abl_{m}", cfg, steps, 3, torch.device("cuda"), 1, 0, with_e2e=False)
+            st = r["stages_ms"]
+            print(f"| {m} | {'KV' if kv else 'KO'} | {mode} | {r['launches_per_step']} | {st['k1_prescan']:.4f} | "
+                  f"{st['k2_scan']:.4f} | {st['k3_postscan']:.4f} | {st['sum_without_pdl']:.4f} | "
+                  f"{r['value']:.1f} |", flush=True)

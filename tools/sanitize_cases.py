@@ -15,6 +15,7 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import oracle  # noqa: E402
+import workloads as W  # noqa: E402
 from msutil import from_dev, make_case, to_dev  # noqa: E402
 import paper_conf_ppopp_ashkianidmo16_b200 as P  # noqa: E402
 from paper_conf_ppopp_ashkianidmo16_b200.dist import scatter_multisplit_virtual  # noqa: E402
@@ -22,8 +23,9 @@ from paper_conf_ppopp_ashkianidmo16_b200.dist import scatter_multisplit_virtual 
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 3 * 4096 * 148 + 77  # > 1 tile per resident CTA, ragged
 cases = [("delta", 8, False, "one"), ("delta", 8, True, "one"), ("splitters", 32, False, "one"),
          ("ids", 32, True, "one"), ("lowbits", 16, True, "ranged"), ("splitters", 32, True, "ranged"),
-         ("delta", 32, False, "3k"), ("ids", 5, True, "3k"), ("delta", 256, False, None),
-         ("splitters", 200, True, None), ("ids", 100, False, None)]
+         ("delta", 32, False, "3k"), ("ids", 5, True, "3k"), ("delta", 256, False, "3k"),
+         ("splitters", 200, True, "3k"), ("ids", 100, False, "3k"), ("delta", 256, True, "ranged"),
+         ("splitters", 100, False, "ranged")]
 fails = 0
 for kind, m, kv, variant in cases:
     case = make_case(kind, m, n, seed=m + 3, kv=kv, dist="binomial")
@@ -54,5 +56,18 @@ for kv in (False, True):  # fused sharded scatter, 3 virtual ranks
     ok = np.array_equal(from_dev(k2), eko) and (evo is None or np.array_equal(from_dev(v2), evo))
     fails += not ok
     print(f"fused scatter P=3 kv={kv:d}: {'ok' if ok else 'MISMATCH'}", flush=True)
+for kind, m, kw, kv in (("delta", 1000, dict(delta=4000037), True), ("ids", 4096, dict(id_bytes=4), False)):
+    # m > 256: two passes + the offsets kernel
+    ospec = oracle.Spec(kind, m, delta=kw.get("delta", 1), id_bytes=kw.get("id_bytes", 1))
+    keys = W.keys_np(n, 5)
+    ids = W.bucket_draw_np(n, 5, "binomial", m).astype(np.uint32) if kind == "ids" else None
+    vals = W.values_np(n, 5, "index") if kv else None
+    plan = P.Plan(P.BucketSpec(kind, m, **kw), n, with_values=kv)
+    ko, vo, off = plan.run(to_dev(keys), to_dev(vals), to_dev(ids))
+    eko, evo, eoff = oracle.multisplit(ospec, keys, vals, ids=ids)
+    ok = np.array_equal(from_dev(ko), eko) and (evo is None or np.array_equal(from_dev(vo), evo)) and \
+        np.array_equal(from_dev(off).astype(np.uint64), eoff)
+    fails += not ok
+    print(f"wide {kind} m={m} kv={kv:d}: launches={plan.last_launches()} {'ok' if ok else 'MISMATCH'}", flush=True)
 print("SANITIZE_CASES", "FAIL" if fails else "OK", flush=True)
 sys.exit(1 if fails else 0)
