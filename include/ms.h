@@ -15,17 +15,13 @@
  *   K2 scan       G = exclusive scan of row-vectorised H, offsets = G[:,0]
  *   K3 post-scan  recompute ids, stable tile-local multisplit in shared
  *                 memory, coalesced scatter to G[j][l] + local offset
- * Variants (ms_plan_geometry reports tile (0), ranged (1), ONE (2), two-pass (3);
+ * Variants (ms_plan_geometry reports tile (0), ranged (1) or ONE (2);
  * ms_plan_last_launches how many kernels the last ms_run enqueued):
  *   "tile"   subproblems = the L tiles (H, G are m x L words): K1, K2, K3;
  *   "ranged" subproblems = the C <= 1024 contiguous tile ranges of K3's
  *            persistent CTAs: K1 writes per-range histograms (C x k x m), K3
  *            folds their scan into its prologue and keeps each tile's G_j as a
- *            running sum inside its range (Eq. (2) applied twice): 2 kernels
- *            (the default for m <= 16 key-value and 32 < m <= 256 runs of
- *            >= 8 tiles per SM);
- *   "two-pass" (m > 256, variant 3): two stable multisplits by the low and
- *            the high digit of the id, then the offsets from the output;
+ *            running sum inside its range (Eq. (2) applied twice): 2 kernels;
  *   "ONE"    (m <= 32; every key-only run and key-value runs of up to 64
  *            tiles per SM) the ranged form in ONE cooperative launch: range
  *            counts, grid barrier, range scan, post-scan (reverse tile walk)
@@ -95,7 +91,7 @@ typedef struct ms_plan_s *ms_plan_t;
  * (m, n, key-only / key-value) by the measured rule of DESIGN.md §7; a
  * MS_VARIANT_* flag makes every run use that one (at most one may be set):
  *   MS_VARIANT_3K      tile variant  K1 -> K2 -> K3     (3 launches, any m)
- *   MS_VARIANT_RANGED  CTA ranges    K1r -> K3          (2 launches, any m <= 256)
+ *   MS_VARIANT_RANGED  CTA ranges    K1r -> K3          (2 launches, m <= 32)
  *   MS_VARIANT_ONE     cooperative   one kernel         (1 launch,  m <= 32; a
  *                      grid that cannot be co-resident fails with MS_ERR_CUDA
  *                      instead of falling back to the ranged variant)
@@ -123,7 +119,7 @@ typedef struct ms_plan_s *ms_plan_t;
  * MS_LOWBITS, delta >= 1, sorted splitters, id_bytes) and the flags, and
  * precomputes the bucket-function constants.  Returns MS_ERR_INVALID_ARG on a
  * bad spec or flag combination, MS_ERR_UNSUPPORTED for a variant the spec
- * cannot use (m > 32 with MS_VARIANT_ONE; m > 256 with any flag but MS_VALIDATE). */
+ * cannot use (m > 32 with MS_VARIANT_RANGED / MS_VARIANT_ONE). */
 ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n,
                          int with_values, uint32_t flags, int device);
 

@@ -115,9 +115,10 @@ Geometry geometry(const ms_plan_s *p, uint64_t n) {
   g.off_hg = kAlign;
   g.off_status = g.off_hg + align_up(g.hg_words * 4);
   g.bytes = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);
-  // the range counts (ranged / ONE variants) reuse the tile arrays' space (never live together)
-  g.off_hc = g.off_hg;
-  g.bytes = std::max(g.bytes, g.off_hc + align_up((size_t)kMaxRangeRows * p->spec.m * 4));
+  if (p->spec.m <= 32) {  // the range counts reuse the tile arrays' space (never live together)
+    g.off_hc = g.off_hg;
+    g.bytes = std::max(g.bytes, g.off_hc + align_up((size_t)kMaxRangeRows * p->spec.m * 4));
+  }
   return g;
 }
 
@@ -233,12 +234,8 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
 }
 
 // K1r: k sub-ranges per range so that the grid has ~8 CTAs of 256 threads per SM
-// K1r: k sub-ranges per range so that the grid has ~8 CTAs of 256 threads per SM; for m > 32
-// (64 KB of byte counters per CTA) at most 2, which keeps the range scan every K3 CTA runs in
-// its prologue at <= 2C rows of m words
 uint32_t k1r_split(const ms_plan_s *p, uint32_t C) {
-  const uint32_t k = std::max<uint32_t>(1u, std::min<uint32_t>(8u * (uint32_t)p->sms / C, kMaxRangeRows / C));
-  return p->spec.m > 32 ? std::min<uint32_t>(k, 2u) : k;
+  return std::max<uint32_t>(1u, std::min<uint32_t>(8u * (uint32_t)p->sms / C, kMaxRangeRows / C));
 }
 
 template <int KIND>
@@ -273,11 +270,8 @@ cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, cons
 // keys; NSkv-like m4..16 KV 321 vs 305 with ONE), the tile variant for 16 < m <= 32 (shorter
 // runs: concurrently processed tiles write ADJACENT runs of every bucket).
 int choose_variant(const ms_plan_s *p, uint64_t L, bool kv) {
-  if (p->direct) return V_TILE;
+  if (p->spec.m > 32 || p->direct) return V_TILE;
   if (p->forced >= 0) return p->forced;
-  // 32 < m <= 256: the ballot K3, per tile (K1 -> K2 -> K3) or over CTA ranges (K1r -> K3: no m x L
-  // H/G arrays, no K2) once the input spans >= 8 tiles per SM
-  if (p->spec.m > 32) return L >= 8ull * (uint64_t)p->sms ? V_RANGED : V_TILE;
   if (!kv || L <= 64ull * (uint64_t)p->sms) return V_ONE;
   if (p->k3nt * p->kpt >= 256u * p->spec.m && L >= 8ull * (uint64_t)p->sms) return V_RANGED;
   return V_TILE;
@@ -558,7 +552,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (vf & (vf - 1)) return MS_ERR_INVALID_ARG;  // at most one variant flag
   if (af & (af - 1)) return MS_ERR_INVALID_ARG;  // at most one ablation
   if (af && vf) return MS_ERR_INVALID_ARG;
-  if ((flags & MS_VARIANT_ONE) && m > 32) return MS_ERR_UNSUPPORTED;
+  if ((flags & (MS_VARIANT_RANGED | MS_VARIANT_ONE)) && m > 32) return MS_ERR_UNSUPPORTED;
   BucketParams bp;
   memset(&bp, 0, sizeof(bp));
   int kkind = spec->kind;

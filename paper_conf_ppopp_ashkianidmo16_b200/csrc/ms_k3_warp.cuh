@@ -23,7 +23,7 @@ namespace ms {
 // (Eq. (2) one level down).  Keys (and values) arrive by one TMA
 // bulk copy per array (UBLKCP) on an mbarrier.
 template <int KIND, bool KV, int R, int LOGM, bool FULL>
-__device__ __forceinline__ uint32_t k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
+__device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
                                         uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
                                         uint64_t base, uint32_t nt, const BucketParams &p,
                                         uint32_t *keys_s, uint32_t *vals_s, uint32_t *cnt_s,
@@ -151,7 +151,6 @@ __device__ __forceinline__ uint32_t k3_tile(const uint32_t *__restrict__ vals_g,
   } else {
     for (uint32_t i = tid; i < nt; i += kThreads) store(i);
   }
-  return tot;  // this tile's count of bucket tid (0 for tid >= m)
 }
 
 template <int KIND, bool KV, int R, int LOGM>
@@ -212,150 +211,14 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   }
 }
 
-// ============================================================== CTA-range K3 (m > 32)
-// Terms 1+2 of Eq. (2) for range c (the C contiguous tile ranges of this persistent grid are the
-// subproblems, ms_ranged.cuh), from K1r's R = C*k rows of m counts, for m <= NT buckets: thread j
-// sums column j of the rows before c*k (pre_j) and after (the rest of tot_j); a block scan of the
-// totals gives start_j; GB[c][j] = start_j + pre_j (CTA 0 also writes offsets).  `red` = NT/32 + 1
-// words of scratch.  Every thread must call it; returns GB[c][tid] (0 for tid >= m).
-template <int NT>
-__device__ __forceinline__ uint32_t range_base_wide(const RangeScan &rs, uint32_t m, uint32_t c, uint32_t n,
-                                                    uint32_t *red) {
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t cut = c * rs.k;
-  uint32_t pre = 0, post = 0;
-  if (tid < m) {
-    const uint32_t *col = rs.HC + tid;
-    uint32_t r = 0;
-#pragma unroll 8
-    for (; r < cut; ++r) pre += __ldcg(col + (uint64_t)r * m);
-#pragma unroll 8
-    for (; r < rs.R; ++r) post += __ldcg(col + (uint64_t)r * m);
-  }
-  const uint32_t tot = pre + post;
-  const uint32_t incl = warp_incl_scan(tot, lane);
-  if (lane == 31) red[warp] = incl;
-  __syncthreads();
-  uint32_t wpre = 0;
-#pragma unroll
-  for (int w = 0; w < NT / 32; ++w) wpre += (w < (int)warp) ? red[w] : 0u;
-  const uint32_t start = wpre + incl - tot;
-  if (c == 0 && rs.offsets != nullptr) {
-    if (tid < m) rs.offsets[tid] = start;
-    if (tid == 0) rs.offsets[m] = n;
-  }
-  __syncthreads();
-  return tid < m ? start + pre : 0u;
-}
-
-// Persistent CTA-range form of the ballot K3 (the ranged variant for 32 < m <= 256): CTA c walks
-// the tiles of range c in order, keys (and values) TMA-staged two tiles ahead, and keeps each
-// bucket's G for the current tile as a running sum (thread j: bucket j) -- no m x L H/G arrays, no
-// K2 launch (DESIGN.md §7 "ranged variant for m > 32").
-template <int KIND, bool KV, int R, int LOGM>
-__global__ void __launch_bounds__(kThreads, 2)
-k3w_ranged(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals, const void *__restrict__ ids,
-           uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n, uint32_t L,
-           const __grid_constant__ BucketParams p, const __grid_constant__ RangeScan rs) {
-  constexpr int T = kThreads * R;
-  extern __shared__ __align__(128) uint8_t smem_raw[];
-  uint32_t *stk = reinterpret_cast<uint32_t *>(smem_raw);  // [2][T] staged keys
-  uint32_t *stv = stk + 2 * T;                              // [2][T] staged values
-  uint32_t *cnt_s = stv + (KV ? 2 * T : 0);                 // [8][256] per-warp counters
-  uint32_t *gD_s = cnt_s + kWarps * kMaxM;                  // [256]
-  uint32_t *spl_s = gD_s + kMaxM;                           // [256]
-  uint32_t *red = spl_s + kMaxM;                            // [16]
-  uint8_t *id8_s = reinterpret_cast<uint8_t *>(red + 16);   // [T]
-  __shared__ __align__(8) uint64_t bar[2];
-  __shared__ uint32_t wsum[kWarps];
-
-  const uint32_t tid = threadIdx.x;
-  const uint32_t m = p.m;
-  const uint64_t r0 = (uint64_t)blockIdx.x * L / gridDim.x;
-  const uint32_t iters = (uint32_t)((uint64_t)(blockIdx.x + 1) * L / gridDim.x - r0);
-  const uint64_t Lfull = n / T;
-  auto issue = [&](uint32_t it) {  // one thread: TMA of tile r0 + it into stage it & 1 (full tiles only)
-    const uint64_t tile = r0 + it;
-    if (it >= iters || tile >= Lfull) return;
-    const uint32_t st = it & 1u;
-    mbar_arrive_expect_tx(&bar[st], (KV ? 2u : 1u) * T * 4u);
-    bulk_g2s(stk + st * T, keys + tile * T, T * 4u, &bar[st]);
-    if constexpr (KV) bulk_g2s(stv + st * T, vals + tile * T, T * 4u, &bar[st]);
-  };
-  if (tid == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
-    fence_mbar_init();
-    issue(0);
-    issue(1);
-  }
-  if constexpr (KIND == SPLITTERS) {
-    if (tid < (1u << p.logm)) spl_s[tid] = p.spl[tid];
-  }
-  pdl_wait();  // K1r's range counts are complete (the first tiles' loads above are already in flight)
-  uint32_t grun = range_base_wide<kThreads>(rs, m, blockIdx.x, n, red);
-  for (uint32_t it = 0; it < iters; ++it) {
-    const uint64_t tile = r0 + it;
-    const uint64_t base = tile * T;
-    const bool full = tile < Lfull;
-    const uint32_t nt = full ? (uint32_t)T : (uint32_t)(n - base);
-    uint32_t *keys_s = stk + (it & 1u) * T, *vals_s = stv + (it & 1u) * T;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] = 0;  // kThreads == kMaxM
-    if (!full) {
-      for (uint32_t i = tid; i < nt; i += kThreads) {
-        keys_s[i] = keys[base + i];
-        if constexpr (KV) vals_s[i] = vals[base + i];
-      }
-    }
-    __syncthreads();
-    uint32_t tot;
-    if (full) {
-      mbar_wait(&bar[it & 1u], (it >> 1) & 1u);
-      tot = k3_tile<KIND, KV, R, LOGM, true>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
-                                             spl_s, id8_s, wsum, grun);
-    } else {
-      tot = k3_tile<KIND, KV, R, LOGM, false>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s,
-                                              gD_s, spl_s, id8_s, wsum, grun);
-    }
-    grun += tot;
-    __syncthreads();  // every thread's stores have read this stage: refill it
-    if (tid == 0) issue(it + 2);
-  }
-}
-
 // ------------------------------------------------------------------ host launcher (m > 32)
 inline size_t k3w_smem(int R, bool kv, bool id8) {
   const size_t T = 256u * R;
   return T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
 }
 
-inline size_t k3w_ranged_smem(int R, bool kv) {
-  const size_t T = 256u * R;
-  return 2 * T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM + 16) * 4 + T;
-}
-
-template <int KIND, bool KV, int R, int LOGM>
-inline cudaError_t k3w_launch_ranged(const K3pArgs &a) {
-  auto k = k3w_ranged<KIND, KV, R, LOGM>;
-  const size_t smem = k3w_ranged_smem(R, KV);
-  cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, smem);
-  if (per_sm <= 0) per_sm = 1;
-  const unsigned grid = (unsigned)umin64_host(umin64_host(a.L, (uint64_t)a.sms * per_sm), kMaxRanges);
-  if (a.grid_out) {
-    *a.grid_out = grid;
-    return cudaSuccess;
-  }
-  const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(grid), dim3(kThreads), smem, a.stream, a.keys, a.vals, a.ids,
-                                  a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rs);
-  return e != cudaSuccess ? e : cudaGetLastError();
-}
-
 template <int KIND, bool KV, int R, int LOGM>
 inline cudaError_t k3w_launch_l(const K3pArgs &a) {
-  if (a.ranged) return k3w_launch_ranged<KIND, KV, R, LOGM>(a);
   constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC && KIND != SHIFT);
   // ballot ranks (__match_any_sync measured 1.6x slower at m = 256 on B200: MATCH.ANY is
   // ADU-bound)

@@ -73,7 +73,7 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t *spl_s = smem;                                              // kMaxM words (SPLITTERS)
   uint32_t *tbl_s = smem + kMaxM;                                      // kSplBins words (SPLITTERS)
-  uint32_t *acc = smem + (KIND == SPLITTERS ? kMaxM + kSplBins : 0);   // [kMaxM]
+  uint32_t *acc = smem + (KIND == SPLITTERS ? kMaxM + kSplBins : 0);   // [32]
   uint8_t *c8 = reinterpret_cast<uint8_t *>(acc + 32);                // [m][NT1]
   const uint32_t tid = threadIdx.x, lane = tid & 31;
   const uint32_t m = p.m;
@@ -83,7 +83,7 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   pdl_trigger();  // K3 (launched with PDL) may be scheduled once every K1r CTA has started
   uint4 *c4 = reinterpret_cast<uint4 *>(c8);
   for (uint32_t i = tid; i < m * (NT1 / 16); i += NT1) c4[i] = make_uint4(0, 0, 0, 0);
-  for (uint32_t i = tid; i < (uint32_t)kMaxM; i += NT1) acc[i] = 0;
+  if (tid < 32) acc[tid] = 0;
   if constexpr (KIND == SPLITTERS) {
     for (uint32_t i = tid; i < (1u << p.logm); i += NT1) spl_s[i] = p.spl[i];
     __syncthreads();
@@ -171,11 +171,11 @@ k1r_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
     if (p.validate && __any_sync(0xFFFFFFFFu, bad) && lane == 0) atomicOr(err_flag, 1u);
   }
   k1r_flush<NT1>(c8, acc, m);
-  for (uint32_t j = tid; j < m; j += NT1) HC[(uint64_t)blockIdx.x * m + j] = acc[j];
+  if (tid < m) HC[(uint64_t)blockIdx.x * m + tid] = acc[tid];
 }
 
 inline size_t k1r_smem(uint32_t m, int kind, int nt1) {
-  return (kind == SPLITTERS ? (kMaxM + kSplBins) * 4 : 0) + kMaxM * 4 + (size_t)m * nt1;
+  return (kind == SPLITTERS ? (kMaxM + kSplBins) * 4 : 0) + 32 * 4 + (size_t)m * nt1;
 }
 
 // Rows of K1r's range-count matrix: R = C * k <= max(C, 8 * SMs) on B200 (<= 1184).

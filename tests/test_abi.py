@@ -71,7 +71,8 @@ def test_plan_create_accepts(spec):
 
 
 @pytest.mark.parametrize("spec,flags", [
-    (BucketSpec("delta", 64, delta=1 << 26), 8),   # ONE needs m <= 32
+    (BucketSpec("delta", 64, delta=1 << 26), 4),   # ranged / ONE need m <= 32
+    (BucketSpec("delta", 64, delta=1 << 26), 8),
     (BucketSpec("delta", 8, delta=5), 16),         # Direct ablation: DELTA with m * delta = 2^32 only
     (BucketSpec("delta", 64, delta=1 << 26), 16),
     (BucketSpec("ids", 8), 16),
@@ -110,8 +111,7 @@ def test_variant_rule():
     assert _variant(d8, 1 << 25, 1) == ONE and _variant(d32, 1 << 25, 1) == ONE   # 8192 tiles <= 64 * 148
     assert _variant(d8, 1 << 28, 1) == RANGED and _variant(d32, 1 << 28, 1) == TILE
     assert _variant(BucketSpec("ids", 16), 1 << 28, 1) == RANGED
-    assert _variant(d256, 1 << 20, 0) == T and _variant(d256, 1 << 28, 1) == RANGED   # >= 8 tiles per SM
-    assert _variant(d256, 1 << 28, 0, 2) == T and _variant(d256, 1 << 20, 1, 4) == RANGED
+    assert _variant(d256, 1 << 20, 0) == T and _variant(d256, 1 << 28, 1) == T
     for flags, want in ((2, TILE), (4, RANGED), (8, ONE)):
         assert _variant(d8, 1 << 28, 1, flags) == want and _variant(d32, 1000, 0, flags) == want
     assert _variant(d8, 1 << 20, 0, 16) == TILE      # the Direct ablation runs the tile variant

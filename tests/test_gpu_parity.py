@@ -69,10 +69,11 @@ NS = [0, 1, 31, 2047, 2048, 2049, 4095, 4097, 8191, 8193, 100003]
 MS = [1, 2, 3, 5, 8, 31, 32, 33, 64, 127, 255, 256]
 
 
-# Low-bit buckets need a power-of-two m (reading #10); ONE is m <= 32 only.
+# Low-bit buckets need a power-of-two m (reading #10); m > 32 always uses the tile variant, so the
+# forced CTA-range and ONE variants are only generated for m <= 32.
 MATRIX = [(kind, m, variant) for variant in (None, "3k", "ranged", "one")
           for kind in ("lowbits", "delta", "splitters", "ids")
-          for m in MS if not (kind == "lowbits" and m & (m - 1)) and not (variant == "one" and m > 32)]
+          for m in MS if not (kind == "lowbits" and m & (m - 1)) and not (variant in ("ranged", "one") and m > 32)]
 
 
 @pytest.mark.parametrize("kind,m,variant", MATRIX)
@@ -136,7 +137,7 @@ def test_parity_distributions(kind, m, dist):
     """Skewed workloads (§6.5): binomial, 75 % hot bucket, all in one bucket."""
     for n in (4097, (1 << 20) + 7):
         case = make_case(kind, m, n, seed=7 + m, dist=dist, kv=True)
-        for variant in ([None, "3k", "ranged", "one"] if m <= 32 else [None, "3k", "ranged"]):
+        for variant in ([None, "3k", "ranged", "one"] if m <= 32 else [None, "3k"]):
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} {dist} n={n} {variant}")
 
 
@@ -472,25 +473,6 @@ def test_wide_validate_flags_out_of_range_ids():
     bad[12345] = 1000
     plan.run(to_dev(keys), ids=to_dev(bad))
     assert plan.check() == -8
-
-
-@pytest.mark.parametrize("kind,m,kv", [("delta", 256, False), ("delta", 256, True), ("splitters", 100, True),
-                                       ("ids", 200, False), ("lowbits", 64, True), ("delta", 33, False)])
-def test_parity_ranged_wide_m(kind, m, kv):
-    """32 < m <= 256 over CTA ranges (K1r -> persistent ballot K3, 2 launches): around the range
-    boundaries (L = C +- 1 ... 13C + 7, ragged last tile) and at the default switch-over."""
-    sms = torch.cuda.get_device_properties(0).multi_processor_count
-    T = 4096
-    for i, L in enumerate([sms - 1, 2 * sms + 1, 8 * sms, 13 * sms + 7]):
-        for n in (L * T, L * T - T + 3):
-            case = make_case(kind, m, n, seed=500 + i, kv=kv, dist="binomial" if i % 2 else "uniform")
-            _assert_equal(case, _run_case(case, "ranged"), _expect(case), f"ranged {kind} m={m} L={L} n={n}")
-    # the default variant takes the ranged path from 8 tiles per SM on
-    n = 8 * sms * T + 5
-    case = make_case(kind, m, n, seed=77, kv=kv)
-    _assert_equal(case, _run_case(case, expect_variant=1), _expect(case), f"default ranged {kind} m={m}")
-
-
 @pytest.mark.parametrize("variant", ["nw2", "nw4"])
 @pytest.mark.parametrize("m", [2, 4, 8, 16, 32])
 def test_parity_nw_ablation(variant, m):

@@ -27,7 +27,11 @@ def _dijkstra(g, source):
 def test_delta_stepping_matches_dijkstra(V, E, wmax, delta, m):
     from paper_conf_ppopp_ashkianidmo16_b200.sssp import delta_stepping, synthetic_graph
     g = synthetic_graph(V, E, wmax, seed=V + E + delta, device="cuda")
-    dist, stats = delta_stepping(g, 0, delta, m)
     exp = _dijkstra(g, 0)
+    dist, stats = delta_stepping(g, 0, delta, m)
     assert np.array_equal(dist.cpu().numpy(), exp)
     assert stats["multisplits"] == stats["iterations"] > 0
+    # the sort-based re-bucketing it replaces (stable: the same buckets in the same order)
+    dist2, stats2 = delta_stepping(g, 0, delta, m, rebucket="sort")
+    assert np.array_equal(dist2.cpu().numpy(), exp)
+    assert stats2["iterations"] == stats["iterations"] and stats2["relaxed_edges"] == stats["relaxed_edges"]

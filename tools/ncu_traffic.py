@@ -16,12 +16,18 @@ METRICS = "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum"
 
 
 def capture(name):
-    cmd = [NCU, "--metrics", METRICS, "--clock-control", "none", "--kernel-name", "regex:^k[123]",
-           "--csv", "--page", "raw", sys.executable, os.path.join(ROOT, "tools", "run_one.py"), name, "2"]
+    cmd = [NCU, "--metrics", METRICS, "--clock-control", "none", "--kernel-name", "regex:^k",
+           "--csv", "--page", "raw", "--print-units", "base", sys.executable, os.path.join(ROOT, "tools", "run_one.py"),
+           name, "2"]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=1800)
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith('"')]
     rows = list(csv.DictReader(io.StringIO("\n".join(lines))))
-    rows = [x for x in rows if x.get("Kernel Name", "").startswith("k")]
+    def base_name(s):
+        s = s.strip()
+        if s.startswith("void "):
+            s = s[5:]
+        return s.split("<")[0].split("(")[0].strip()
+    rows = [x for x in rows if base_name(x.get("Kernel Name", "")).startswith("k")]
     if not rows:
         sys.stderr.write(r.stdout[-2000:] + r.stderr[-2000:])
         return None
@@ -31,9 +37,9 @@ def capture(name):
         def num(k):
             return float(str(x[k]).replace(",", ""))
         rd, wr = num("dram__bytes_read.sum"), num("dram__bytes_write.sum")
-        unit_r = x.get("dram__bytes_read.sum_unit") if "dram__bytes_read.sum_unit" in x else None
-        out.append({"kernel": x["Kernel Name"].split("(")[0].strip(), "dram_read": rd, "dram_write": wr,
-                    "dram_bytes": rd + wr, "time_ns": num("gpu__time_duration.sum"), "unit_hint": unit_r})
+        out.append({"kernel": base_name(x["Kernel Name"]), "instance": x["Kernel Name"].split("(")[0].strip(),
+                    "dram_read": rd, "dram_write": wr, "dram_bytes": rd + wr,
+                    "time_ns": num("gpu__time_duration.sum")})
     return out
 
 
