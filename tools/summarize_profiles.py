@@ -1,5 +1,5 @@
 """Summarise a round's ncu artefacts into profiles/: python tools/summarize_profiles.py r01
-Writes profiles/<tag>_summary.md and updates profiles/ncu_traffic.json (K3 dram bytes per launch)."""
+Writes profiles/<tag>_summary.md (profiles/ncu_traffic.json is written by tools/ncu_traffic.py)."""
 import csv
 import io
 import json
@@ -50,8 +50,6 @@ if os.path.exists(lp):
 
 # (2) full captures
 PROF_OUT = os.environ.get("PROF_OUT", os.path.join(ROOT, "profiles"))
-traffic_path = os.path.join(PROF_OUT, "ncu_traffic.json")
-traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
 keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__issue_active.avg.pct_of_peak_sustained_active",
         "sm__warps_active.avg.pct_of_peak_sustained_active", "l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed",
@@ -78,11 +76,12 @@ for f in sorted(os.listdir(src)):
     wr, wru = get("dram__bytes_write.sum")
     dram = to_bytes(rd, rdu) + to_bytes(wr, wru)
     c = bench.CONFIGS[cfg]
-    pre, post = model.pass_bytes_per_key(c["kv"])
+    pre, post = model.pass_bytes_per_key(c["kv"], 1 if c["kind"] == "ids" else 0)
     alg = (post if kern.startswith("k3") else pre if kern.startswith("k1") else 0) * c["n"]
-    # the library's ONE rule (ms_api.cu): m <= 32 key-only, or key-value up to 64
-    # tiles per SM, runs K1 + K3 in one cooperative k3v_postscan launch -> 12 / 20 B per key
-    one = kern == "k3v_postscan" and c["m"] <= 32 and (not c["kv"] or c["n"] // 4096 <= 64 * 148)
+    # the library's own variant choice (ms_plan_geometry): ONE runs K1 + K3 in one cooperative
+    # k3v_postscan launch -> all of the step's bytes
+    from paper_conf_ppopp_ashkianidmo16_b200 import Plan
+    one = kern == "k3v_postscan" and Plan(bench.spec_of(c), c["n"], with_values=c["kv"]).geometry(c["n"])[2] == 2
     if one:
         alg = (pre + post) * c["n"]
     stalls = [(hh.replace("smsp__average_warps_issue_stalled_", "").replace("_per_issue_active.ratio", ""),
@@ -98,10 +97,6 @@ for f in sorted(os.listdir(src)):
             out.append(f"- {k}: {v:g} {un}")
     out.append("- top stalls (cycles per issued instruction): " + ", ".join(f"{a} {b:.2f}" for a, b in stalls[:6]))
     out.append("")
-    if kern.startswith("k3"):
-        traffic[cfg] = int(dram)
-with open(traffic_path, "w") as fh:
-    json.dump(traffic, fh, indent=1, sort_keys=True)
 os.makedirs(PROF_OUT, exist_ok=True)
 with open(os.path.join(PROF_OUT, f"{tag}_summary.md"), "w") as fh:
     fh.write(f"# ncu summary, round tag {tag}\n\nGenerated by tools/summarize_profiles.py from "
