@@ -22,3 +22,12 @@ cap C4ko k2_scan
 cap C3 k3v_postscan
 cap IDSko k3v_postscan
 ls gpurun_out | grep prof_${TAG}
+# summarise on the box (the .ncu-rep files are too large to bring back): text summaries only
+PROF_OUT=gpurun_out python tools/summarize_profiles.py ${TAG} > /dev/null 2>&1
+for f in gpurun_out/prof_${TAG}_*.ncu-rep; do
+  b=$(basename $f .ncu-rep)
+  python tools/ncu_summary.py $f > gpurun_out/${b}_metrics.txt 2>&1
+  python tools/ncu_lines.py $f 40 > gpurun_out/${b}_lines.txt 2>&1
+done
+mkdir -p /tmp/ncu_reps && mv gpurun_out/prof_${TAG}_*.ncu-rep /tmp/ncu_reps/ 2>/dev/null
+ls gpurun_out | grep ${TAG}
