@@ -173,27 +173,6 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   // c[j][beta] at shared address ccol + j * RS
   const uint32_t ccol = smem_u32(cnt) + 2 * beta + 16 * (beta >> 6);
   const uint32_t ks32 = smem_u32(keys_s), vs32 = smem_u32(vals_s);
-  // Stable ranks of 4 consecutive keys of this thread's block in its private counter column
-  // (term 3 of Eq. (2) one level down): the 4 counters are read first -- one shared-memory round
-  // trip per group instead of 4 dependent read-modify-writes -- duplicates inside the group are
-  // resolved by id compares, and the increments are stored in key order (a later store to the same
-  // counter carries the larger value).  Returns the 4 ranks as bytes; keys j >= nvalid are skipped.
-  auto rmw4 = [&](const uint32_t (&id)[4], int nvalid) -> uint32_t {
-    uint32_t a[4], l[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      a[j] = ccol + id[j] * RS;
-      l[j] = j < nvalid ? lds_u16(a[j]) : 0u;
-    }
-    const uint32_t r0 = l[0], r1 = l[1] + (id[1] == id[0]);
-    const uint32_t r2 = l[2] + (id[2] == id[0]) + (id[2] == id[1]);
-    const uint32_t r3 = l[3] + (id[3] == id[0]) + (id[3] == id[1]) + (id[3] == id[2]);
-    const uint32_t r[4] = {r0, r1, r2, r3};
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (j < nvalid) sts_u16(a[j], r[j] + 1);
-    return r0 | (r1 << 8) | (r2 << 16) | (r3 << 24);
-  };
 
   const uint64_t r0 = RANGED ? (uint64_t)blockIdx.x * L / gridDim.x : 0;
   const uint32_t iters = RANGED ? (uint32_t)((uint64_t)(blockIdx.x + 1) * L / gridDim.x - r0)
@@ -302,8 +281,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     auto cnt4 = [&](const uint4 *x) {
 #pragma unroll
       for (int c = 0; c < NCH; ++c) {
-        const uint32_t id[4] = {id_of(x[c].x), id_of(x[c].y), id_of(x[c].z), id_of(x[c].w)};
-        rmw4(id, 4);
+        count1(x[c].x); count1(x[c].y); count1(x[c].z); count1(x[c].w);
       }
     };
     if constexpr (P1TMA) {
@@ -331,8 +309,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
           load_ids_full(tb + (uint64_t)(IDB == 1 ? 16 : 4) * (c * NT + tid), w, IDB == 1 ? 4 : 1);
 #pragma unroll
           for (int q = 0; q < (IDB == 1 ? 4 : 1); ++q) {
-            const uint32_t id[4] = {w[q] & 255u, (w[q] >> 8) & 255u, (w[q] >> 16) & 255u, w[q] >> 24};
-            rmw4(id, 4);
+            count_id(w[q] & 255u); count_id((w[q] >> 8) & 255u);
+            count_id((w[q] >> 16) & 255u); count_id(w[q] >> 24);
           }
         }
         if ((sq & 2047u) == 2047u) fold();
@@ -447,15 +425,21 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 #pragma unroll
     for (int c = 0; c < NCH; ++c) {
       const uint32_t kk[4] = {kx[c].x, kx[c].y, kx[c].z, kx[c].w};
-      uint32_t id[4];
+      rk[c] = 0u;
+      if constexpr (KEEP_ID && KIND != IDS) idk[c] = 0u;
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        if constexpr (KIND == IDS) id[j] = __byte_perm(idk[c], 0u, 0x4440u + j);
-        else id[j] = id_of(kk[j]);
+        if (FULL || b0 + 4 * c + j < nt) {
+          uint32_t id;
+          if constexpr (KIND == IDS) id = __byte_perm(idk[c], 0u, 0x4440u + j);
+          else id = id_of(kk[j]);
+          const uint32_t a = ccol + id * RS;
+          const uint32_t r = lds_u16(a);
+          sts_u16(a, r + 1);
+          rk[c] |= r << (8 * j);
+          if constexpr (KEEP_ID && KIND != IDS) idk[c] |= id << (8 * j);
+        }
       }
-      const int nv = FULL ? 4 : (int)min(4u, nt > b0 + 4 * c ? nt - (b0 + 4 * c) : 0u);
-      rk[c] = rmw4(id, nv);
-      if constexpr (KEEP_ID && KIND != IDS) idk[c] = id[0] | (id[1] << 8) | (id[2] << 16) | (id[3] << 24);
     }
     __syncthreads();
     // the key stage is free again (keys are in registers): refill it
