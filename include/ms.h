@@ -15,17 +15,22 @@
  *   K2 scan       G = exclusive scan of row-vectorised H, offsets = G[:,0]
  *   K3 post-scan  recompute ids, stable tile-local multisplit in shared
  *                 memory, coalesced scatter to G[j][l] + local offset
- * Variants (ms_plan_geometry reports tile (0), ranged (1) or ONE (2);
- * ms_plan_last_launches how many kernels the last ms_run enqueued):
- *   "tile"   subproblems = the L tiles (H, G are m x L words): K1, K2, K3;
- *   "ranged" subproblems = the C <= 1024 contiguous tile ranges of K3's
- *            persistent CTAs: K1 writes per-range histograms (C x k x m), K3
- *            folds their scan into its prologue and keeps each tile's G_j as a
- *            running sum inside its range (Eq. (2) applied twice): 2 kernels;
- *   "ONE"    (m <= 32; every key-only run and key-value runs of up to 64
- *            tiles per SM) the ranged form in ONE cooperative launch: range
- *            counts, grid barrier, range scan, post-scan (reverse tile walk)
- *            -- 1 kernel.  DESIGN.md §7.
+ * Variants (ms_plan_geometry reports tile (0), ranged (1), ONE (2) or
+ * two-pass (3); ms_plan_last_launches how many kernels the last ms_run
+ * enqueued):
+ *   "tile"   subproblems = the L tiles (H, G are m x L words): K1, K2, K3
+ *            (the default for 32 < m <= 256);
+ *   "ranged" (m <= 32) subproblems = the C <= 1024 contiguous tile ranges of
+ *            K3's persistent CTAs: K1 writes per-range histograms (C x k x m),
+ *            K3 folds their scan into its prologue and keeps each tile's G_j as
+ *            a running sum inside its range (Eq. (2) applied twice): 2 kernels
+ *            (the default for key-value runs of >= 8 (m <= 8), >= 16 (m <= 16,
+ *            MS_IDS) or > 64 (m <= 32) tiles per SM);
+ *   "ONE"    (m <= 32; every other run) the ranged form in ONE cooperative
+ *            launch: range counts, grid barrier, range scan, post-scan
+ *            (reverse tile walk) -- 1 kernel.  DESIGN.md §7-8;
+ *   "two-pass" (m > 256) two stable multisplits by the low and the high digit
+ *            of the id, then the offsets from the sorted output (§7b).
  * Every variant computes the same (unique, stable) result.  The MS_VARIANT_*
  * plan flags force one.  The stage-wise calls (ms_prescan / ms_scan /
  * ms_postscan) always use tiles.

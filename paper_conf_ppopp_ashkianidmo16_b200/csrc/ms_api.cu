@@ -263,18 +263,18 @@ cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, cons
   }
 }
 
-// The variant a run of L tiles uses (measured on B200).  m > 32 and the Direct
-// ablation: tile.  Forced by a MS_VARIANT_* plan flag: that one.  Otherwise ONE for every
-// key-only run and for key-value runs of up to 64 tiles per SM (C3, n = 2^25: 192 -> 207
-// G keys/s); above that the CTA-range variant for m <= 16 (mean bucket run per tile >= 256
-// keys; NSkv-like m4..16 KV 321 vs 305 with ONE), the tile variant for 16 < m <= 32 (shorter
-// runs: concurrently processed tiles write ADJACENT runs of every bucket).
+// The variant a run of L tiles uses (measured on B200 with tools/variant_sweep.py,
+// profiles/r02_variants.md).  m > 32 and the Direct ablation: tile.  Forced by a MS_VARIANT_* plan
+// flag: that one.  Key-only: ONE (m32 KO at 2^27: 407 vs 400 ranged vs 390 tile).  Key-value: the
+// CTA-range variant once the input spans enough tiles per SM -- >= 8 for m <= 8 (m2 KV at 2^25:
+// 294 vs 283 ONE), >= 16 for m <= 16 and precomputed ids (IDS m=32 KV at 2^25: 236 vs 224),
+// > 64 above (C3 at 2^27: 234 vs 232 ONE vs 224 tile; at 2^25 ONE 212 vs 205) -- ONE below.
 int choose_variant(const ms_plan_s *p, uint64_t L, bool kv) {
   if (p->spec.m > 32 || p->direct) return V_TILE;
   if (p->forced >= 0) return p->forced;
-  if (!kv || L <= 64ull * (uint64_t)p->sms) return V_ONE;
-  if (p->k3nt * p->kpt >= 256u * p->spec.m && L >= 8ull * (uint64_t)p->sms) return V_RANGED;
-  return V_TILE;
+  if (!kv) return V_ONE;
+  const uint64_t per_sm = p->spec.m <= 8 ? 8 : (p->spec.m <= 16 || p->kkind == IDS) ? 16 : 65;
+  return L >= per_sm * (uint64_t)p->sms ? V_RANGED : V_ONE;
 }
 
 ms_status check_ws(const ms_plan_s *p, uint64_t n, void *ws, size_t ws_bytes, Geometry *g) {

@@ -101,16 +101,18 @@ def _variant(spec, n, kv, flags=0):
 
 
 def test_variant_rule():
-    """ms_plan_geometry reports the variant the run takes: ONE for key-only m <= 32 and
-    for key-value up to 64 tiles per SM, then ranged (m <= 16) or tile (m > 16); tile for m > 32;
-    a MS_VARIANT_* flag always wins.  (Without a GPU the SM count is B200's 148.)"""
+    """ms_plan_geometry reports the variant the run takes (DESIGN.md §8): ONE for key-only m <= 32;
+    key-value: ranged from 8 (m <= 8), 16 (m <= 16, precomputed ids) or 65 (m <= 32) tiles per SM,
+    ONE below; tile for m > 32; a MS_VARIANT_* flag always wins.  (Without a GPU the SM count is
+    B200's 148.)"""
     T, ONE, RANGED, TILE = _abi.VARIANT_TILE, _abi.VARIANT_ONE, _abi.VARIANT_RANGED, _abi.VARIANT_TILE
     d8, d32, d256 = (BucketSpec("delta", 8, delta=1 << 29), BucketSpec("delta", 32, delta=1 << 27),
                      BucketSpec("delta", 256, delta=1 << 24))
     assert _variant(d8, 1 << 28, 0) == ONE and _variant(d32, 1 << 28, 0) == ONE
-    assert _variant(d8, 1 << 25, 1) == ONE and _variant(d32, 1 << 25, 1) == ONE   # 8192 tiles <= 64 * 148
-    assert _variant(d8, 1 << 28, 1) == RANGED and _variant(d32, 1 << 28, 1) == TILE
-    assert _variant(BucketSpec("ids", 16), 1 << 28, 1) == RANGED
+    assert _variant(d8, 1 << 25, 1) == RANGED and _variant(d32, 1 << 25, 1) == ONE  # 8192 tiles: 55 per SM
+    assert _variant(d8, 1 << 22, 1) == ONE and _variant(d8, 1 << 23, 1) == RANGED   # 1024 / 2048 tiles
+    assert _variant(d8, 1 << 28, 1) == RANGED and _variant(d32, 1 << 28, 1) == RANGED
+    assert _variant(BucketSpec("ids", 32), 1 << 25, 1) == RANGED and _variant(BucketSpec("ids", 32), 1 << 23, 1) == ONE
     assert _variant(d256, 1 << 20, 0) == T and _variant(d256, 1 << 28, 1) == T
     for flags, want in ((2, TILE), (4, RANGED), (8, ONE)):
         assert _variant(d8, 1 << 28, 1, flags) == want and _variant(d32, 1000, 0, flags) == want

@@ -107,10 +107,10 @@ def test_ranged_range_edges(kind, m, kv, variant):
 @pytest.mark.parametrize("kind,m", [("delta", 2), ("delta", 8), ("lowbits", 16), ("splitters", 16), ("ids", 8),
                                     ("delta", 32), ("ids", 32)])
 def test_parity_default_large_kv(kind, m, n):
-    """The library's DEFAULT key-value path above 64 tiles per SM: K1r -> K3 (2 launches) for
-    m <= 16, K1 -> K2 -> K3 (3 launches) for 16 < m <= 32 -- at n = 2^26 + 5 and 2^28, full compare."""
+    """The library's DEFAULT key-value path at n = 2^26 + 5 and 2^28 (K1r -> K3, 2 launches), full
+    compare."""
     case = make_case(kind, m, n, seed=900 + m, kv=True, vals_kind="random")
-    want = _abi_mod().VARIANT_RANGED if m <= 16 else _abi_mod().VARIANT_TILE
+    want = _abi_mod().VARIANT_RANGED
     _assert_equal(case, _run_case(case, expect_variant=want), _expect(case), f"default KV {kind} m={m} n={n}")
 
 
