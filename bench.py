@@ -71,6 +71,11 @@ for _m in (2, 4, 8, 16, 32, 64, 128, 256):
             desc=f"{'key-value' if _kv else 'key-only'} m={_m} delta D=2^32/m, n=2^28, uniform", kind="delta",
             m=_m, delta=(1 << 32) // _m, n=1 << 28, kv=_kv, dist="uniform", seed=W.SEEDS["C4"])
 
+for _m in (512, 1024, 4096, 16384, 65536):  # m > 256 (two-pass plans; the Fig. 4 question)
+    for _kv in (False, True):
+        CONFIGS[f"wide_m{_m}_{'kv' if _kv else 'ko'}"] = dict(
+            desc=f"{'key-value' if _kv else 'key-only'} m={_m} delta D=2^32/m, n=2^28, uniform", kind="delta",
+            m=_m, delta=(1 << 32) // _m, n=1 << 28, kv=_kv, dist="uniform", seed=W.SEEDS["C4"])
 for _e in (22, 23, 24, 26, 27, 28):  # size sweep of C2 (fixed-cost analysis)
     CONFIGS[f"C2_n{_e}"] = dict(CONFIGS["C2"], n=1 << _e, desc=CONFIGS["C2"]["desc"].replace("2^25", f"2^{_e}"))
 for _d, _dn in (("binomial", "bin"), ("hot", "hot")):  # skewed north-star workloads (Fig. 5)
@@ -87,12 +92,14 @@ CONFIGS["IDSkv"] = dict(desc="key-value m=32 precomputed u8 ids, n=2^28, uniform
 CONFIGS["C5"] = dict(desc="sharded key-value m=32 splitter buckets, n=2^31 total (strong-scaled over the GPUs), "
                           "uniform", kind="splitters", m=32, n=1 << 31, kv=True, dist="uniform",
                      seed=W.SEEDS.get("C5", 0x4D530005), strong=True)
+CONFIGS["C5s"] = dict(CONFIGS["C5"], n=1 << 26, desc=CONFIGS["C5"]["desc"].replace("2^31", "2^26 (small C5, tests)"))
 
 DEFAULT = "NSko"      # N = 1 headline
 DEFAULT_DIST = "C5"   # N > 1 headline
 EXTRA_DEFAULT = ",".join(["NSkv", "NSbin_ko", "NShot_ko", "NSbin_kv", "NShot_kv", "C4ko", "C4kv", "C3", "C3bin",
                           "C3hot", "C2", "C2far", "C1", "IDSko", "IDSkv"] +
-                         [f"sweep_m{m}_{t}" for t in ("ko", "kv") for m in (2, 4, 8, 16, 64, 128)])
+                         [f"sweep_m{m}_{t}" for t in ("ko", "kv") for m in (2, 4, 8, 16, 64, 128)] +
+                         [f"wide_m{m}_{t}" for t in ("ko", "kv") for m in (512, 4096, 65536)])
 
 
 def log(*a):
@@ -457,8 +464,10 @@ def measure_comparators(cfg, plan, keys, vals, ids, K, flush):
             return sk, vals[idx]
         return sk, None
 
-    def reduced_bit():
-        b = torch_bucket_ids(cfg, keys, ids).to(torch.uint8 if cfg["m"] <= 256 else torch.int32)
+    def reduced_bit():  # the fewest id bits torch can sort: u8 (m <= 256), or i16 of id - 2^15 (m <= 65536)
+        b = torch_bucket_ids(cfg, keys, ids)
+        b = b.to(torch.uint8) if cfg["m"] <= 256 else (b - 32768).to(torch.int16) if cfg["m"] <= 65536 else \
+            b.to(torch.int32)
         _, idx = torch.sort(b, stable=True)
         return keys[idx], (vals[idx] if vals is not None else None)
 
@@ -494,9 +503,6 @@ def measure_comparators(cfg, plan, keys, vals, ids, K, flush):
     return out
 
 
-KERNEL_OF_VARIANT = {0: "k3", 1: "k3v_postscan", 2: "k3v_postscan"}
-
-
 def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparators=False):
     import torch
     import paper_conf_ppopp_ashkianidmo16_b200 as P
@@ -521,10 +527,11 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparato
     T, L, variant = plan.geometry(n)
     alg_bytes = model.algorithmic_bytes_per_key(cfg["kv"], idb) * n
     one = launches == 1  # ONE cooperative launch: the single kernel moves all 12 (KO) / 20 (KV) B per key
-    kern_bytes = alg_bytes if one else post_b * n
-    kern_ms = k3_ms
+    wide = variant == 3  # m > 256: two passes + offsets; reported as a whole against the one-pass model
+    kern_bytes = alg_bytes if (one or wide) else post_b * n
+    kern_ms = ms_step if wide else k3_ms
     achieved = kern_bytes / (kern_ms * 1e-3) / 1e9
-    kname = ("k3v_postscan" if cfg["m"] <= 32 else "k3_postscan")
+    kname = "two-pass plan" if wide else ("k3v_postscan" if cfg["m"] <= 32 else "k3_postscan")
     wl = np.array(whole)
     res = {
         "value": value, "ms_per_step": ms_step,
@@ -538,16 +545,16 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparato
         "whole_step_frac_nominal_8tbs": alg_bytes / (ms_step * 1e-3) / 1e9 / NOMINAL_HBM_GBS,
         "roofline": {"bound": "hbm",
                      "kernel": (kname + " ONE (pre-scan + scan + post-scan in one cooperative launch)") if one
-                     else kname + " (post-scan)",
+                     else kname + " (whole step vs the one-pass byte model)" if wide else kname + " (post-scan)",
                      "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4),
                      "frac_vs_nominal_8tbs": round(achieved / NOMINAL_HBM_GBS, 4),
                      "traffic": load_traffic(name, kname),
                      "algorithmic_bytes_per_launch": kern_bytes,
                      "algorithmic_bytes_per_key": kern_bytes / n,
                      "peak_source": peak_src,
-                     "k1_prescan_frac": None if one else round(pre_b * n / (k1_ms * 1e-3) / 1e9 / peak, 4)},
+                     "k1_prescan_frac": None if (one or wide) else round(pre_b * n / (k1_ms * 1e-3) / 1e9 / peak, 4)},
         "gpu_launches": launches * K, "launches_per_step": launches, "tile": T, "tiles": L,
-        "variant": ["tile", "ranged", "one"][variant], "clocks": clocks.result(),
+        "variant": ["tile", "ranged", "one", "two-pass"][variant], "clocks": clocks.result(),
     }
     if comparators:
         comp = measure_comparators(cfg, plan, keys, vals, ids, 3, flush)
@@ -695,8 +702,14 @@ def run_ours(args, name, cfg, world, rank, local):
     # one process per GPU; ranks beyond the visible GPUs share them (only for the gloo test mode)
     device = torch.device("cuda", local % max(1, torch.cuda.device_count()))
     torch.cuda.set_device(device)
-    if world > 1:
+    sharded = world > 1 or args.sharded_at_1
+    if sharded:
         import torch.distributed as dist
+        if world == 1:  # --sharded-at-1: the N > 1 code path on a one-rank process group (testing)
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", "29517")
+            os.environ.setdefault("RANK", "0")
+            os.environ.setdefault("WORLD_SIZE", "1")
         if args.dist_backend == "nccl":
             dist.init_process_group("nccl", device_id=device)
         else:
@@ -705,7 +718,7 @@ def run_ours(args, name, cfg, world, rank, local):
     if rank == 0:
         b.build()
     barrier(world)
-    if world == 1:
+    if not sharded:
         res = bench_config(name, cfg, args.steps, args.warmup, device, world, rank, with_e2e=True,
                            comparators=not args.no_extra)
     else:
@@ -764,7 +777,7 @@ def run_ours(args, name, cfg, world, rank, local):
             if k in res:
                 out[k] = res[k]
         print(json.dumps(out), flush=True)
-    if world > 1:
+    if sharded:
         import torch.distributed as dist
         dist.destroy_process_group()
 
@@ -782,6 +795,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N>1 exchange backend (gloo: host-staged, for testing on one GPU)")
+    ap.add_argument("--sharded-at-1", action="store_true",
+                    help="run the N > 1 sharded code path (NCCL communicator, ms_dist_run) on one GPU (testing)")
     ap.add_argument("--dist-mode", default="nccl", choices=["nccl", "fused"],
                     help="N>1 exchange: ms_dist_run (NCCL send/recv after a local ms_run), or the fused K3 that "
                          "stores into the owners' symmetric-memory windows (m <= 32, computed bucket ids)")
