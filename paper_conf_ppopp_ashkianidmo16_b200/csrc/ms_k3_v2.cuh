@@ -358,6 +358,17 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 
   // one tile; FULL (compile time): all T keys valid, TMA-staged.  The partial
   // tile (at most one, the last of its CTA) is peeled off the loop
+  // MS_IDS with u8 ids: the next full tile's 16 ids of this thread are loaded one tile ahead
+  // (a register double buffer), so their HBM latency overlaps a whole tile instead of stalling the
+  // counting pass
+  uint4 idpre = make_uint4(0, 0, 0, 0);
+  auto id_prefetch = [&](uint32_t it) {
+    if constexpr (KIND == IDS && IDB == 1) {
+      if (it < iters && tile_of(it) < Lfull)
+        idpre = __ldcs(reinterpret_cast<const uint4 *>(static_cast<const uint8_t *>(ids) + tile_of(it) * T + b0));
+    }
+  };
+  id_prefetch(ONE ? ptail : 0u);  // the first full tile of the walk
   auto tile_body = [&](uint32_t it, auto fullc) {
     constexpr bool FULL = decltype(fullc)::value;
     const uint64_t tile = tile_of(it);
@@ -410,7 +421,10 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     uint32_t rk[NCH];                   // ranks (< K), one byte each
     uint32_t idk[KEEP_ID ? NCH : 1];    // kept ids, one byte each
     if constexpr (KIND == IDS) {
-      if constexpr (FULL) {
+      if constexpr (FULL && IDB == 1) {
+        idk[0] = clamp4(idpre.x); idk[1] = clamp4(idpre.y); idk[2] = clamp4(idpre.z); idk[3] = clamp4(idpre.w);
+        id_prefetch(it + 1);
+      } else if constexpr (FULL) {
         load_ids_full(base + b0, idk, 4);
       } else {
 #pragma unroll
