@@ -99,7 +99,7 @@ struct Geometry {
   uint64_t L;
   uint64_t hg_words;   // m * L
   uint64_t chunks;     // K2 CTAs
-  size_t off_hg, off_status, off_flag, bytes;
+  size_t off_hg, off_status, off_flag, off_rowtot, bytes;
   size_t off_hc;          // CTA-range / ONE variants: range counts HC[R][m], over the H/G region
 };
 
@@ -114,7 +114,8 @@ Geometry geometry(const ms_plan_s *p, uint64_t n) {
   g.off_flag = 0;
   g.off_hg = kAlign;
   g.off_status = g.off_hg + align_up(g.hg_words * 4);
-  g.bytes = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);
+  g.off_rowtot = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);  // m > 32: K2's row totals
+  g.bytes = g.off_rowtot + align_up((size_t)kMaxM * 4);
   if (p->spec.m <= 32) {  // the range counts reuse the tile arrays' space (never live together)
     g.off_hc = g.off_hg;
     g.bytes = std::max(g.bytes, g.off_hc + align_up((size_t)kMaxRangeRows * p->spec.m * 4));
@@ -200,7 +201,8 @@ cudaError_t dispatch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *k
 cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *keys,
                         const uint32_t *vals, const void *ids, const uint32_t *G, uint32_t *ko,
                         uint32_t *vo, uint32_t n, uint32_t *flag, cudaStream_t s, int ranged = 0,
-                        uint32_t *grid_out = nullptr, int pdl = 0, const RangeScan *rs = nullptr) {
+                        uint32_t *grid_out = nullptr, int pdl = 0, const RangeScan *rs = nullptr,
+                        const uint32_t *rowtot = nullptr) {
   K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
             p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, p->sms, s};
   a.ranged = ranged;
@@ -208,6 +210,7 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   a.pdl = pdl;
   a.direct = p->direct;
   a.flag = flag;
+  a.rowtot = rowtot;
   if (rs) a.rs = *rs;
   if (p->spec.m <= 32) {  // K3 v2 (ms_k3_v2.cuh), one TU per kind
     switch (p->kkind) {
@@ -877,19 +880,30 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
     p->last_launches = 2;
     return MS_OK;
   }
-  cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, status, (uint32_t)g.chunks, flag, s);
+  // m > 32: K2 row by row (k2w_rowscan, no look-back; term 1 of Eq. (2) folded into K3)
+  const bool rowk2 = p->spec.m > 32;
+  uint32_t *rowtot = (uint32_t *)(w + g.off_rowtot);
+  cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, rowk2 ? nullptr : status,
+                              rowk2 ? 0u : (uint32_t)g.chunks, flag, s);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev && p->tracing == 1) cudaEventRecord(ev[1], s);
-  if (launch_ex(pdl, k2_scan, dim3((unsigned)g.chunks), dim3(kThreads), 0, s, HG, (uint64_t)g.hg_words, status,
-                offsets, (uint32_t)g.L, p->spec.m, (uint32_t)n) != cudaSuccess ||
-      cudaGetLastError() != cudaSuccess)
+  if (rowk2) {
+    if (launch_ex(pdl, k2w_rowscan, dim3(p->spec.m), dim3(kRowThreads), 0, s, HG, (uint32_t)g.L, rowtot) !=
+            cudaSuccess ||
+        cudaGetLastError() != cudaSuccess)
+      return MS_ERR_CUDA;
+  } else if (launch_ex(pdl, k2_scan, dim3((unsigned)g.chunks), dim3(kThreads), 0, s, HG, (uint64_t)g.hg_words,
+                       status, offsets, (uint32_t)g.L, p->spec.m, (uint32_t)n) != cudaSuccess ||
+             cudaGetLastError() != cudaSuccess) {
     return MS_ERR_CUDA;
+  }
   if (ev && p->tracing == 1) cudaEventRecord(ev[2], s);
   // K3 after the many-CTA K2 of the tile variant: PDL only for key-only runs
   // (measured: an early-resident key-value K3 -- 2 CTAs with
   // the whole register file per SM -- costs ~6 % at n = 2^28)
+  const RangeScan rso{nullptr, offsets, 0, 0};  // m > 32: K3 CTA 0 writes the offsets
   e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, flag, s, 0, nullptr,
-                  pdl && vals_in == nullptr);
+                  pdl && vals_in == nullptr, rowk2 ? &rso : nullptr, rowk2 ? rowtot : nullptr);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev) cudaEventRecord(ev[3], s);
   p->last_launches = 3;

@@ -455,6 +455,70 @@ k2_scan(uint32_t *__restrict__ data, uint64_t total, uint64_t *__restrict__ stat
   if (offsets != nullptr && chunk == 0 && tid == 0) offsets[m] = n;
 }
 
+// ============================================================== K2, row-parallel (m > 32)
+// The same terms 1+2 of Eq. (2) split into their two sums: CTA j scans bucket row j of H alone
+// (term 2: G'[j][l] = sum_{l'<l} h_{j,l'}, in place) and writes the row total; term 1 (the
+// exclusive scan of the m row totals) is left to K3, whose CTAs each scan the m totals once
+// (k3_postscan's `rowtot` mode).  No look-back chain: m independent CTAs stream their rows
+// (32 KB chunks staged in shared memory with a running carry), against the chained single-pass
+// scan of m*L words that the look-back serialises (C4: 72 us).
+constexpr int kRowThreads = 512;
+constexpr int kRowItems = 16;
+constexpr int kRowChunk = kRowThreads * kRowItems;  // 8192 words
+
+__global__ void __launch_bounds__(kRowThreads)
+k2w_rowscan(uint32_t *__restrict__ HG, uint32_t L, uint32_t *__restrict__ rowtot) {
+  __shared__ uint32_t buf[kRowChunk + kRowChunk / 32];
+  __shared__ uint32_t wsum[kRowThreads / 32];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  uint32_t *row = HG + (uint64_t)blockIdx.x * L;
+  pdl_wait();  // K1's H is complete and visible
+  pdl_trigger();
+  uint32_t carry = 0;
+  for (uint32_t base = 0; base < L; base += kRowChunk) {
+    const uint32_t cnt = min(L - base, (uint32_t)kRowChunk);
+#pragma unroll
+    for (int j = 0; j < kRowItems; ++j) {
+      const uint32_t i = j * kRowThreads + tid;
+      buf[i + (i >> 5)] = i < cnt ? __ldcs(row + base + i) : 0u;
+    }
+    __syncthreads();
+    uint32_t v[kRowItems], s = 0;
+#pragma unroll
+    for (int q = 0; q < kRowItems; ++q) {
+      const uint32_t i = tid * kRowItems + q;
+      v[q] = buf[i + (i >> 5)];
+      s += v[q];
+    }
+    const uint32_t incl = warp_incl_scan(s, lane);
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    uint32_t wpre = 0, agg = 0;
+#pragma unroll
+    for (int w = 0; w < kRowThreads / 32; ++w) {
+      const uint32_t x = wsum[w];
+      wpre += (w < (int)warp) ? x : 0u;
+      agg += x;
+    }
+    uint32_t run = carry + wpre + incl - s;
+#pragma unroll
+    for (int q = 0; q < kRowItems; ++q) {
+      const uint32_t i = tid * kRowItems + q;
+      buf[i + (i >> 5)] = run;
+      run += v[q];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < kRowItems; ++j) {
+      const uint32_t i = j * kRowThreads + tid;
+      if (i < cnt) __stcg(row + base + i, buf[i + (i >> 5)]);
+    }
+    carry += agg;
+    __syncthreads();  // buf and wsum are reused by the next chunk
+  }
+  if (tid == 0) rowtot[blockIdx.x] = carry;
+}
+
 // ============================================================== whatBucket() only
 template <int KIND>
 __global__ void __launch_bounds__(kThreads)
