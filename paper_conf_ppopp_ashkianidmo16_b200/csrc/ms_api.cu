@@ -114,8 +114,9 @@ Geometry geometry(const ms_plan_s *p, uint64_t n) {
   g.off_flag = 0;
   g.off_hg = kAlign;
   g.off_status = g.off_hg + align_up(g.hg_words * 4);
-  g.off_rowtot = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);  // m > 32: K2's row totals
-  g.bytes = g.off_rowtot + align_up((size_t)kMaxM * 4);
+  // m > 32: K2's row totals [kMaxM], row bases [kMaxM] and its ticket
+  g.off_rowtot = g.off_status + align_up(std::max<uint64_t>(g.chunks, 1) * 8);
+  g.bytes = g.off_rowtot + align_up((size_t)(2 * kMaxM + 2) * 4);
   if (p->spec.m <= 32) {  // the range counts reuse the tile arrays' space (never live together)
     g.off_hc = g.off_hg;
     g.bytes = std::max(g.bytes, g.off_hc + align_up((size_t)kMaxRangeRows * p->spec.m * 4));
@@ -882,14 +883,15 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   }
   // m > 32: K2 row by row (k2w_rowscan, no look-back; term 1 of Eq. (2) folded into K3)
   const bool rowk2 = p->spec.m > 32;
-  uint32_t *rowtot = (uint32_t *)(w + g.off_rowtot);
-  cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, rowk2 ? nullptr : status,
-                              rowk2 ? 0u : (uint32_t)g.chunks, flag, s);
+  uint32_t *rowtot = (uint32_t *)(w + g.off_rowtot), *rowbase = rowtot + kMaxM, *ticket = rowbase + kMaxM;
+  // K1 zeroes K2's look-back status words, or (row K2) its 8-byte ticket word
+  cudaError_t e = dispatch_k1(p, g, keys_in, ids, (uint32_t)n, HG, rowk2 ? (uint64_t *)ticket : status,
+                              rowk2 ? 1u : (uint32_t)g.chunks, flag, s);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev && p->tracing == 1) cudaEventRecord(ev[1], s);
   if (rowk2) {
-    if (launch_ex(pdl, k2w_rowscan, dim3(p->spec.m), dim3(kRowThreads), 0, s, HG, (uint32_t)g.L, rowtot) !=
-            cudaSuccess ||
+    if (launch_ex(pdl, k2w_rowscan, dim3(p->spec.m), dim3(kRowThreads), 0, s, HG, (uint32_t)g.L, p->spec.m,
+                  (uint32_t)n, rowtot, rowbase, ticket, offsets) != cudaSuccess ||
         cudaGetLastError() != cudaSuccess)
       return MS_ERR_CUDA;
   } else if (launch_ex(pdl, k2_scan, dim3((unsigned)g.chunks), dim3(kThreads), 0, s, HG, (uint64_t)g.hg_words,
@@ -901,9 +903,8 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
   // K3 after the many-CTA K2 of the tile variant: PDL only for key-only runs
   // (measured: an early-resident key-value K3 -- 2 CTAs with
   // the whole register file per SM -- costs ~6 % at n = 2^28)
-  const RangeScan rso{nullptr, offsets, 0, 0};  // m > 32: K3 CTA 0 writes the offsets
   e = dispatch_k3(p, g, keys_in, vals_in, ids, HG, keys_out, vals_out, (uint32_t)n, flag, s, 0, nullptr,
-                  pdl && vals_in == nullptr, rowk2 ? &rso : nullptr, rowk2 ? rowtot : nullptr);
+                  pdl && vals_in == nullptr, nullptr, rowk2 ? rowbase : nullptr);
   if (e != cudaSuccess) return MS_ERR_CUDA;
   if (ev) cudaEventRecord(ev[3], s);
   p->last_launches = 3;

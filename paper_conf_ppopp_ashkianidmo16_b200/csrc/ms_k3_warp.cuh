@@ -158,10 +158,9 @@ __global__ void __launch_bounds__(kThreads)
 k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
             const void *__restrict__ ids, const uint32_t *__restrict__ G,
             uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
-            uint32_t L, const __grid_constant__ BucketParams p, const uint32_t *__restrict__ rowtot,
-            uint32_t *__restrict__ offsets) {
-  // G: the full Eq. (2) terms 1+2 (K2 = k2_scan), or -- rowtot != nullptr (K2 = k2w_rowscan) --
-  // term 2 only, row by row, with term 1 = the exclusive scan of the m row totals, computed here
+            uint32_t L, const __grid_constant__ BucketParams p, const uint32_t *__restrict__ rowbase) {
+  // G: the full Eq. (2) terms 1+2 (K2 = k2_scan), or -- rowbase != nullptr (K2 = k2w_rowscan) --
+  // term 2 only, row by row, with term 1 in rowbase[j]
   constexpr int T = kThreads * R;
   extern __shared__ __align__(128) uint8_t smem_raw[];
   uint32_t *keys_s = reinterpret_cast<uint32_t *>(smem_raw);
@@ -198,22 +197,7 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   uint32_t gcol = 0;
   pdl_wait();  // K2's G is complete (the tile's TMA load above is already in flight)
   if (tid < m) gcol = __ldg(G + (uint64_t)tid * L + tile);
-  if (rowtot != nullptr) {  // term 1: exclusive scan of the row totals (kThreads == kMaxM >= m)
-    const uint32_t lane = tid & 31, warp = tid >> 5;
-    const uint32_t t = tid < m ? __ldg(rowtot + tid) : 0u;
-    const uint32_t incl = warp_incl_scan(t, lane);
-    if (lane == 31) wsum[warp] = incl;
-    __syncthreads();
-    uint32_t start = incl - t;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) start += (w < (int)warp) ? wsum[w] : 0u;
-    gcol += start;
-    if (tile == 0 && offsets != nullptr) {
-      if (tid < m) offsets[tid] = start;
-      if (tid == 0) offsets[m] = n;
-    }
-    __syncthreads();  // wsum is reused by the tile
-  }
+  if (rowbase != nullptr && tid < m) gcol += __ldg(rowbase + tid);
 #pragma unroll
   for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] = 0;  // kThreads == kMaxM
   if constexpr (KIND == SPLITTERS) {
@@ -245,7 +229,7 @@ inline cudaError_t k3w_launch_l(const K3pArgs &a) {
   const size_t smem = k3w_smem(R, KV, id8);
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(a.L), dim3(kThreads), smem, a.stream, a.keys, a.vals, a.ids,
-                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rowtot, a.rs.offsets);
+                                  a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rowtot);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

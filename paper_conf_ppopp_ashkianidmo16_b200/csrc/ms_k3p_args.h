@@ -51,7 +51,7 @@ struct K3pArgs {
   const DistTarget *ds = nullptr;           // fused sharded scatter (K3 v2, tile variant only)
   int direct = 0;                           // ablation: K3 v2 without the local reorder (MS_ABLATION_DIRECT)
   uint32_t *flag = nullptr;                 // IDS + validation: set to 1 when some id >= m
-  const uint32_t *rowtot = nullptr;         // m > 32: G holds row-local scans, term 1 from these row totals
+  const uint32_t *rowtot = nullptr;         // m > 32: G holds row-local scans, term 1 in rowtot[j] (row base)
 };
 
 // Launch with cudaLaunchAttributeProgrammaticStreamSerialization when `pdl`:

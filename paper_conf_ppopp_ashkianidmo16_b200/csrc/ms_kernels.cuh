@@ -457,19 +457,22 @@ k2_scan(uint32_t *__restrict__ data, uint64_t total, uint64_t *__restrict__ stat
 
 // ============================================================== K2, row-parallel (m > 32)
 // The same terms 1+2 of Eq. (2) split into their two sums: CTA j scans bucket row j of H alone
-// (term 2: G'[j][l] = sum_{l'<l} h_{j,l'}, in place) and writes the row total; term 1 (the
-// exclusive scan of the m row totals) is left to K3, whose CTAs each scan the m totals once
-// (k3_postscan's `rowtot` mode).  No look-back chain: m independent CTAs stream their rows
-// (32 KB chunks staged in shared memory with a running carry), against the chained single-pass
-// scan of m*L words that the look-back serialises (C4: 72 us).
+// (term 2: G'[j][l] = sum_{l'<l} h_{j,l'}, in place) and writes the row total; the last CTA to
+// finish (atomic ticket, zeroed by K1) scans the m row totals -- term 1, rowbase[j] =
+// sum_{k<j} tot_k -- and writes the offsets; K3 adds rowbase[j] to G'[j][tile] (k3_postscan's
+// `rowbase` mode).  No look-back chain: m independent CTAs stream their rows (32 KB chunks staged
+// in shared memory with a running carry), against the chained single-pass scan of m*L words that
+// the look-back serialises (C4: 72 us).
 constexpr int kRowThreads = 512;
 constexpr int kRowItems = 16;
 constexpr int kRowChunk = kRowThreads * kRowItems;  // 8192 words
 
 __global__ void __launch_bounds__(kRowThreads)
-k2w_rowscan(uint32_t *__restrict__ HG, uint32_t L, uint32_t *__restrict__ rowtot) {
+k2w_rowscan(uint32_t *__restrict__ HG, uint32_t L, uint32_t m, uint32_t n, uint32_t *__restrict__ rowtot,
+            uint32_t *__restrict__ rowbase, uint32_t *__restrict__ ticket, uint32_t *__restrict__ offsets) {
   __shared__ uint32_t buf[kRowChunk + kRowChunk / 32];
   __shared__ uint32_t wsum[kRowThreads / 32];
+  __shared__ uint32_t last;
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t *row = HG + (uint64_t)blockIdx.x * L;
   pdl_wait();  // K1's H is complete and visible
@@ -516,7 +519,30 @@ k2w_rowscan(uint32_t *__restrict__ HG, uint32_t L, uint32_t *__restrict__ rowtot
     carry += agg;
     __syncthreads();  // buf and wsum are reused by the next chunk
   }
-  if (tid == 0) rowtot[blockIdx.x] = carry;
+  if (tid == 0) {
+    rowtot[blockIdx.x] = carry;
+    __threadfence();
+    last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  // the last row CTA: term 1 = exclusive scan of the m (<= kRowThreads) row totals
+  __threadfence();
+  const uint32_t t = tid < m ? __ldcg(rowtot + tid) : 0u;
+  const uint32_t incl = warp_incl_scan(t, lane);
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  uint32_t start = incl - t;
+#pragma unroll
+  for (int w = 0; w < kRowThreads / 32; ++w) start += (w < (int)warp) ? wsum[w] : 0u;
+  if (tid < m) {
+    rowbase[tid] = start;
+    if (offsets != nullptr) offsets[tid] = start;
+  }
+  if (tid == 0) {
+    if (offsets != nullptr) offsets[m] = n;
+    *ticket = 0;  // (K1 zeroes it again before the next K2)
+  }
 }
 
 // ============================================================== whatBucket() only
