@@ -15,27 +15,33 @@
 
 namespace ms {
 
-// offsets[j] = #{ i : id(src[i]) < j } for j = 0..m, with src sorted by id.  Thread t owns the
-// 4 positions [4t, 4t+4) (one 128-bit load plus the element before them); a position i whose id
-// differs from its predecessor's writes offsets(prev_id, id], the first position writes
-// offsets[0..id], the last writes offsets(id, m].  Every offset is written exactly once.
+// offsets[j] = #{ i : id(src[i]) < j } for j = 0..m, with src sorted by id.  Each thread step
+// owns 16 consecutive positions (four 128-bit loads in flight, plus the element before them); a
+// position i whose id differs from its predecessor's writes offsets(prev_id, id], the first
+// position writes offsets[0..id], the last writes offsets(id, m].  Every offset is written
+// exactly once.
+constexpr int kWideKeys = 16;
 template <int KIND>
 __global__ void __launch_bounds__(256)
 k_wide_offsets(const uint32_t *__restrict__ src, uint64_t n, uint32_t *__restrict__ offsets,
                const __grid_constant__ BucketParams p) {
   const uint32_t m = p.m;
-  for (uint64_t q = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; q * 4 < n; q += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t i0 = q * 4;
-    uint32_t v[4];
-    if (i0 + 4 <= n) {
-      const uint4 x = __ldcs(reinterpret_cast<const uint4 *>(src + i0));
-      v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  for (uint64_t q = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; q * kWideKeys < n;
+       q += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t i0 = q * kWideKeys;
+    uint32_t v[kWideKeys];
+    if (i0 + kWideKeys <= n) {
+#pragma unroll
+      for (int c = 0; c < kWideKeys / 4; ++c) {
+        const uint4 x = __ldcs(reinterpret_cast<const uint4 *>(src + i0) + c);
+        v[4 * c] = x.x; v[4 * c + 1] = x.y; v[4 * c + 2] = x.z; v[4 * c + 3] = x.w;
+      }
     } else {
-      for (int e = 0; e < 4; ++e) v[e] = i0 + e < n ? src[i0 + e] : 0u;
+      for (int e = 0; e < kWideKeys; ++e) v[e] = i0 + e < n ? src[i0 + e] : 0u;
     }
     uint32_t prev = i0 ? bucket_of_key<KIND>(__ldg(src + i0 - 1), p, nullptr) : 0u;
 #pragma unroll
-    for (int e = 0; e < 4; ++e) {
+    for (int e = 0; e < kWideKeys; ++e) {
       const uint64_t i = i0 + e;
       if (i >= n) break;
       const uint32_t id = bucket_of_key<KIND>(v[e], p, nullptr);
@@ -62,7 +68,7 @@ k_ids_check(const uint32_t *__restrict__ ids, uint64_t n, uint32_t m, uint32_t *
 
 cudaError_t wide_offsets_launch(int kind, const uint32_t *src, uint64_t n, uint32_t *offsets,
                                 const BucketParams &bp, int sms, cudaStream_t s) {
-  const unsigned grid = (unsigned)umin64_host((n + 1023) / 1024, (uint64_t)sms * 8);
+  const unsigned grid = (unsigned)umin64_host((n + 256 * kWideKeys - 1) / (256 * kWideKeys), (uint64_t)sms * 8);
   switch (kind) {
     case LOWBITS: k_wide_offsets<LOWBITS><<<grid, 256, 0, s>>>(src, n, offsets, bp); break;
     case SHIFTC: k_wide_offsets<SHIFTC><<<grid, 256, 0, s>>>(src, n, offsets, bp); break;
