@@ -326,6 +326,29 @@ ms_status ms_dist_run(ms_plan_t plan, void *nccl_comm, const uint32_t *keys_in, 
                       uint64_t out_capacity, uint64_t *offsets_global, uint64_t *win_start, uint64_t *win_len,
                       void *workspace, size_t workspace_bytes, void *stream);
 
+/* ---------------------------------------------------------------------------
+ * ms_dist_run_fused -- the same collective with the exchange fused into the
+ * post-scan: local K1 + K2 (ms_prescan / ms_scan), the NCCL
+ * all-gather of the counts (the one host synchronisation), ms_dist_targets,
+ * then ONE post-scan kernel (ms_postscan_scatter) that stores every bucket run
+ * straight into the owning rank's window -- over NVLink / NVSwitch when
+ * keys_windows[r] / vals_windows[r] are peer mappings of rank r's window
+ * buffers (e.g. torch symmetric memory); finally a one-word NCCL all-reduce on
+ * `stream` as the barrier after which every window is complete.  No local
+ * output and no staging copy: 12 / 20 B per key of HBM + NVLink traffic.
+ * keys_windows / vals_windows: HOST arrays of P device pointers valid on this
+ * GPU, each window holding window_capacity elements (MS_ERR_INVALID_ARG if a
+ * window is too small for its balanced share, checked before any store).
+ * m <= 32 and a computed bucket kind (else MS_ERR_UNSUPPORTED); P <=
+ * MS_MAX_PEERS.  Workspace: ms_dist_workspace_size_fused.  Other arguments and
+ * errors as ms_dist_run.
+ * ------------------------------------------------------------------------- */
+ms_status ms_dist_workspace_size_fused(ms_plan_t plan, uint64_t n_local, int32_t nranks, size_t *bytes);
+ms_status ms_dist_run_fused(ms_plan_t plan, void *nccl_comm, const uint32_t *keys_in, const uint32_t *vals_in,
+                            uint64_t n_local, uint32_t *const *keys_windows, uint32_t *const *vals_windows,
+                            uint64_t window_capacity, uint64_t *offsets_global, uint64_t *win_start,
+                            uint64_t *win_len, void *workspace, size_t workspace_bytes, void *stream);
+
 /* NCCL bootstrap for ms_dist_run (the 128-byte unique id travels between the
  * processes by any means, e.g. a torch.distributed broadcast):
  * ms_nccl_get_unique_id writes NCCL_UNIQUE_ID_BYTES (128) bytes to `id` (rank 0);

@@ -36,7 +36,8 @@ EXPORTS = [
     "ms_bucket_ids", "ms_plan_check", "ms_plan_destroy", "ms_status_string",
     "ms_plan_last_launches", "ms_plan_trace", "ms_plan_trace_read", "ms_dist_pieces",
     "ms_dist_targets", "ms_postscan_scatter", "ms_plan_spec", "ms_dist_workspace_size", "ms_dist_run",
-    "ms_nccl_get_unique_id", "ms_nccl_comm_init", "ms_nccl_comm_destroy",
+    "ms_nccl_get_unique_id", "ms_nccl_comm_init", "ms_nccl_comm_destroy", "ms_dist_workspace_size_fused",
+    "ms_dist_run_fused",
 ]
 
 MS_MAX_PEERS = 8
@@ -107,6 +108,9 @@ def lib():
     L.ms_plan_spec.argtypes = [P, ctypes.POINTER(ms_bucket_spec), ctypes.POINTER(I32)]
     L.ms_dist_workspace_size.argtypes = [P, U64, I32, ctypes.POINTER(SZ)]
     L.ms_dist_run.argtypes = [P, P, P, P, P, U64, P, P, U64, P, ctypes.POINTER(U64), ctypes.POINTER(U64), P, SZ, P]
+    L.ms_dist_workspace_size_fused.argtypes = [P, U64, I32, ctypes.POINTER(SZ)]
+    L.ms_dist_run_fused.argtypes = [P, P, P, P, U64, P, P, U64, P, ctypes.POINTER(U64), ctypes.POINTER(U64), P,
+                                    SZ, P]
     L.ms_nccl_get_unique_id.argtypes = [P]
     L.ms_nccl_comm_init.argtypes = [ctypes.POINTER(P), I32, I32, P, ctypes.c_int]
     L.ms_nccl_comm_destroy.argtypes = [P]

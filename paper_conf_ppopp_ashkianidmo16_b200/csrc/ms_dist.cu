@@ -147,6 +147,7 @@ struct Nccl {
   ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
   ncclResult_t (*GroupStart)();
   ncclResult_t (*GroupEnd)();
+  ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t);
 };
 
 const Nccl &nccl() {
@@ -172,6 +173,7 @@ const Nccl &nccl() {
     sym(N.Recv, "ncclRecv");
     sym(N.GroupStart, "ncclGroupStart");
     sym(N.GroupEnd, "ncclGroupEnd");
+    sym(N.AllReduce, "ncclAllReduce");
     N.ok = all;
   });
   return N;
@@ -332,4 +334,126 @@ extern "C" ms_status ms_dist_run(ms_plan_t plan, void *comm, const uint32_t *key
   }
   const ncclResult_t r2 = N.GroupEnd();
   return (r == ncclSuccess && r2 == ncclSuccess) ? MS_OK : MS_ERR_NCCL;
+}
+
+// =========================================================================
+// ms_dist_run_fused: the sharded multisplit with the exchange fused into the
+// post-scan: local K1 + K2 (ms_prescan / ms_scan), the count
+// all-gather, the host targets (ms_dist_targets), then ONE K3 that stores every
+// bucket run straight into the owners' windows (ms_postscan_scatter; TMA bulk
+// stores over NVLink / NVSwitch when the windows are peer mappings), and a
+// one-word NCCL all-reduce on the stream as the barrier after which every
+// window is complete.
+// =========================================================================
+namespace {
+
+struct FusedLayout {
+  size_t local_ws, off_hg, off_loff, off_cnt, off_gath, off_bar, bytes;
+};
+
+FusedLayout fused_layout(ms_plan_t plan, uint32_t m, uint64_t n_local, int nranks, ms_status *st) {
+  FusedLayout d{};
+  size_t ws = 0;
+  uint32_t T = 0;
+  uint64_t L = 0;
+  *st = ms_plan_workspace_size(plan, n_local, &ws);
+  if (*st == MS_OK) *st = ms_plan_geometry(plan, n_local, &T, &L, nullptr);
+  d.local_ws = dalign(ws);
+  d.off_hg = d.local_ws;
+  d.off_loff = d.off_hg + dalign((size_t)m * L * 4);
+  d.off_cnt = d.off_loff + dalign((size_t)(m + 1) * 4);
+  d.off_gath = d.off_cnt + dalign((size_t)m * 8);
+  d.off_bar = d.off_gath + dalign((size_t)nranks * m * 8);
+  d.bytes = d.off_bar + dalign(4);
+  return d;
+}
+
+}  // namespace
+
+extern "C" ms_status ms_dist_workspace_size_fused(ms_plan_t plan, uint64_t n_local, int32_t nranks, size_t *bytes) {
+  if (!plan || !bytes || nranks < 1 || nranks > MS_MAX_PEERS) return MS_ERR_INVALID_ARG;
+  ms_bucket_spec spec;
+  ms_status st = ms_plan_spec(plan, &spec, nullptr);
+  if (st != MS_OK) return st;
+  FusedLayout d = fused_layout(plan, spec.m, n_local, nranks, &st);
+  if (st != MS_OK) return st;
+  *bytes = d.bytes;
+  return MS_OK;
+}
+
+extern "C" ms_status ms_dist_run_fused(ms_plan_t plan, void *comm, const uint32_t *keys_in, const uint32_t *vals_in,
+                                       uint64_t n_local, uint32_t *const *keys_windows,
+                                       uint32_t *const *vals_windows, uint64_t window_capacity,
+                                       uint64_t *offsets_global, uint64_t *win_start, uint64_t *win_len,
+                                       void *workspace, size_t workspace_bytes, void *stream) {
+  if (!plan || !comm || !keys_windows || !workspace) return MS_ERR_INVALID_ARG;
+  ms_bucket_spec spec;
+  int32_t kv = 0;
+  ms_status st = ms_plan_spec(plan, &spec, &kv);
+  if (st != MS_OK) return st;
+  if (vals_in && (!kv || !vals_windows)) return vals_windows ? MS_ERR_UNSUPPORTED : MS_ERR_INVALID_ARG;
+  if (spec.m > 32 || spec.kind == MS_IDS) return MS_ERR_UNSUPPORTED;
+  const Nccl &N = nccl();
+  if (!N.ok) return MS_ERR_NCCL;
+  ncclComm_t c = (ncclComm_t)comm;
+  int P = 0, rank = 0, dev = 0;
+  if (N.CommCount(c, &P) != ncclSuccess || N.CommUserRank(c, &rank) != ncclSuccess ||
+      N.CommCuDevice(c, &dev) != ncclSuccess)
+    return MS_ERR_NCCL;
+  if (P > MS_MAX_PEERS) return MS_ERR_UNSUPPORTED;
+  const uint32_t m = spec.m;
+  FusedLayout d = fused_layout(plan, m, n_local, P, &st);
+  if (st != MS_OK) return st;
+  if (workspace_bytes < d.bytes) return MS_ERR_WORKSPACE;
+  if (reinterpret_cast<uintptr_t>(workspace) & 15u) return MS_ERR_ALIGNMENT;
+  int prev = -1;
+  if (cudaGetDevice(&prev) != cudaSuccess) return MS_ERR_CUDA;
+  if (prev != dev && cudaSetDevice(dev) != cudaSuccess) return MS_ERR_CUDA;
+  struct Restore {
+    int prev, dev;
+    ~Restore() {
+      if (prev != dev) cudaSetDevice(prev);
+    }
+  } restore{prev, dev};
+  cudaStream_t s = (cudaStream_t)stream;
+  char *w = (char *)workspace;
+  uint32_t *HG = (uint32_t *)(w + d.off_hg), *loff = (uint32_t *)(w + d.off_loff), *bar = (uint32_t *)(w + d.off_bar);
+  uint64_t *cnt = (uint64_t *)(w + d.off_cnt), *gath = (uint64_t *)(w + d.off_gath);
+  // 1. local K1 + K2 (tiles; G stays in the workspace for K3)
+  if ((st = ms_prescan(plan, keys_in, nullptr, n_local, HG, workspace, d.local_ws, stream)) != MS_OK) return st;
+  if ((st = ms_scan(plan, HG, n_local, loff, workspace, d.local_ws, stream)) != MS_OK) return st;
+  // 2. counts, all-gathered, on the host
+  k_counts_from_offsets<<<1, 256, 0, s>>>(loff, cnt, m);
+  if (cudaGetLastError() != cudaSuccess) return MS_ERR_CUDA;
+  if (N.AllGather(cnt, gath, m, ncclUint64, c, s) != ncclSuccess) return MS_ERR_NCCL;
+  std::vector<uint64_t> counts((size_t)P * m);
+  if (cudaMemcpyAsync(counts.data(), gath, counts.size() * 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return MS_ERR_CUDA;
+  // 3. targets: global - local position per local bucket, the window starts
+  ms_scatter_target t{};
+  t.nranks = P;
+  if ((st = ms_dist_targets(P, rank, m, counts.data(), t.delta, t.win_start)) != MS_OK) return st;
+  for (int r = 0; r < P; ++r) {
+    if (t.win_start[r + 1] - t.win_start[r] > window_capacity) return MS_ERR_INVALID_ARG;
+    t.keys_dst[r] = keys_windows[r];
+    t.vals_dst[r] = vals_in ? vals_windows[r] : nullptr;
+  }
+  if (offsets_global) {
+    uint64_t B = 0;
+    for (uint32_t b = 0; b < m; ++b) {
+      offsets_global[b] = B;
+      for (int g = 0; g < P; ++g) B += counts[(size_t)g * m + b];
+    }
+    offsets_global[m] = B;
+  }
+  if (win_start) *win_start = t.win_start[rank];
+  if (win_len) *win_len = t.win_start[rank + 1] - t.win_start[rank];
+  // 4. the post-scan storing into the owners' windows
+  if ((st = ms_postscan_scatter(plan, keys_in, vals_in, HG, n_local, &t, workspace, d.local_ws, stream)) != MS_OK)
+    return st;
+  // 5. barrier: every rank's scatter kernel precedes its all-reduce on its stream
+  if (cudaMemsetAsync(bar, 0, 4, s) != cudaSuccess) return MS_ERR_CUDA;
+  if (N.AllReduce == nullptr || N.AllReduce(bar, bar, 1, ncclUint32, ncclSum, c, s) != ncclSuccess) return MS_ERR_NCCL;
+  return MS_OK;
 }

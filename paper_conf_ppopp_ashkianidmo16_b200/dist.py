@@ -189,56 +189,91 @@ def scatter_multisplit_virtual(shards_keys, shards_vals=None, spec=None):
     return keys, vals
 
 
-_SYMM = {}
+class FusedDistPlan:
+    """ms_dist_run_fused (include/ms.h): the sharded multisplit whose post-scan stores every run
+    straight into the owners' windows.  The windows are torch symmetric-memory buffers (allocated
+    and rendezvoused once per plan, mapped on every peer over NVLink / NVSwitch); `peer_windows`
+    overrides them with explicit per-rank device pointers (e.g. virtual ranks on one GPU).
+    m <= 32, computed bucket kinds."""
+
+    def __init__(self, spec, comm: "NcclComm", max_local: int, max_total: int, with_values: bool = False,
+                 group=None, peer_windows=None):
+        import torch
+        from .api import Plan
+        if spec.m > 32 or spec.kind == "ids":
+            raise NotImplementedError("the fused sharded scatter runs on K3 v2 (m <= 32, computed bucket ids)")
+        self.spec, self.comm, self.kv = spec, comm, with_values
+        self.plan = Plan(spec, max(int(max_local), 1), with_values=with_values, device=comm.device)
+        b = ctypes.c_size_t()
+        check(_abi.lib().ms_dist_workspace_size_fused(self.plan._h, max(int(max_local), 1), comm.nranks,
+                                                      ctypes.byref(b)), "ms_dist_workspace_size_fused")
+        dev = torch.device("cuda", comm.device)
+        self.ws = torch.empty(max(b.value, 256), dtype=torch.uint8, device=dev)
+        self.cap = -(-int(max_total) // comm.nranks) + 1
+        if peer_windows is not None:
+            kp, vp = peer_windows
+            self.bufs = None
+        else:
+            import torch.distributed as dist
+            import torch.distributed._symmetric_memory as symm_mem
+            grp = group if group is not None else dist.group.WORLD
+            self.bufs, ptrs = [], []
+            for _ in range(2 if with_values else 1):
+                buf = symm_mem.empty(self.cap, dtype=torch.int32, device=dev)
+                h = symm_mem.rendezvous(buf, grp)
+                self.bufs.append(buf)
+                ptrs.append(list(h.buffer_ptrs))
+            kp, vp = ptrs[0], (ptrs[1] if with_values else None)
+        P = comm.nranks
+        self._kp = (ctypes.c_void_p * P)(*[int(x) for x in kp])
+        self._vp = (ctypes.c_void_p * P)(*[int(x) for x in vp]) if vp is not None else None
+
+    def run(self, keys, vals=None, stream=None, copy_out=True):
+        """Collective.  Returns (keys_window, vals_window, offsets_global u64[m+1] numpy, window_start);
+        the windows are complete on return of the stream's work (the call ends with an NCCL barrier).
+        copy_out=False returns views of this rank's symmetric window (overwritten by the next run)."""
+        from .api import _ptr, _stream
+        offg = np.zeros(self.spec.m + 1, dtype=np.uint64)
+        ws0, wl = ctypes.c_uint64(), ctypes.c_uint64()
+        check(_abi.lib().ms_dist_run_fused(self.plan._h, self.comm._h, _ptr(keys), _ptr(vals), keys.numel(),
+                                           self._kp, self._vp if vals is not None else None, self.cap,
+                                           offg.ctypes.data_as(ctypes.c_void_p), ctypes.byref(ws0), ctypes.byref(wl),
+                                           _ptr(self.ws), self.ws.numel(), _stream(stream)), "ms_dist_run_fused")
+        if self.bufs is None:
+            return None, None, offg, ws0.value
+        k = self.bufs[0][:wl.value]
+        v = self.bufs[1][:wl.value] if vals is not None else None
+        if copy_out:
+            k = k.clone()
+            v = v.clone() if v is not None else None
+        return k, v, offg, ws0.value
+
+
+_FUSED = {}
 
 
 def dist_multisplit_fused(keys, vals=None, spec=None, group=None):
     """Collective, one process per GPU (NCCL process group): like dist_multisplit, but the
-    exchange IS the post-scan kernel: windows are symmetric-memory buffers mapped on every peer
-    (torch.distributed._symmetric_memory over NVLink/NVSwitch) and each rank's K3 stores its
-    runs straight into them.  Returns (keys_window, vals_window, win_start)."""
-    import torch
+    exchange IS the post-scan kernel (ms_dist_run_fused into symmetric-memory windows).  Returns
+    (keys_window, vals_window, window_start); the windows are copies the caller owns."""
     import torch.distributed as dist
-    import torch.distributed._symmetric_memory as symm_mem
     P = dist.get_world_size(group)
-    g = dist.get_rank(group)
-    m = spec.m
-    kv = vals is not None
-    plan = _fused_plan(spec, keys.numel(), kv)
-    ws = plan.workspace(keys.numel())
-    G, cnt = _local_scan(plan, keys, ws)
-    c = torch.as_tensor(cnt.astype(np.int64), device=keys.device)
-    gathered = torch.empty(P * m, dtype=torch.int64, device=keys.device)
-    dist.all_gather_into_tensor(gathered, c, group=group)
-    counts = gathered.cpu().numpy().astype(np.uint64).reshape(P, m)
-    delta, wst = dist_targets(P, g, m, counts)
-    wmax = max(int(wst[r + 1] - wst[r]) for r in range(P)) or 4
-    grp = group if group is not None else dist.group.WORLD
-    # symmetric windows are allocated + rendezvoused once per (group, device, arrays) and reused
-    # while they are large enough (every rank takes the same decision: wmax is global)
-    key = (id(grp), str(keys.device), kv)
-    ent = _SYMM.get(key)
-    if ent is None or ent[0] < wmax:
-        cap = max(wmax, 4)
-        bufs, ptrs = [], []
-        for _ in range(2 if kv else 1):
-            b = symm_mem.empty(cap, dtype=torch.int32, device=keys.device)
-            h = symm_mem.rendezvous(b, grp)
-            bufs.append(b)
-            ptrs.append(list(h.buffer_ptrs))
-        ent = _SYMM[key] = (cap, bufs, ptrs)
-    _, bufs, ptrs = ent
-    t = scatter_target(ptrs[0], ptrs[1] if kv else None, wst, delta)
-    plan.postscan_scatter(keys, G, t, vals=vals, workspace=ws)
-    torch.cuda.current_stream().synchronize()
-    dist.barrier(group)  # every rank's stores into my window are complete
-    wl = int(wst[g + 1] - wst[g])
-    # the symmetric windows are reused by the next call (every rank scatters into them again):
-    # hand the caller tensors it owns
-    out_k = bufs[0][:wl].clone()
-    out_v = bufs[1][:wl].clone() if kv else None
-    dist.barrier(group)  # no rank starts its next scatter into my window before my copy is taken
-    return out_k, out_v, int(wst[g])
+    n = keys.numel()
+    key = (id(group), keys.device.index, vals is not None, spec.kind, spec.m, spec.shift, spec.delta,
+           tuple(spec.splitters or ()))
+    ent = _FUSED.get(key)
+    if ent is None or ent[0] < n:
+        comm = ent[1].comm if ent is not None else NcclComm(group, keys.device.index)
+        # every rank sizes for the largest shard (max over ranks) and the global total
+        import torch
+        t = torch.tensor([n, n], dtype=torch.int64, device=keys.device)
+        dist.all_reduce(t[:1], op=dist.ReduceOp.MAX, group=group)
+        dist.all_reduce(t[1:], op=dist.ReduceOp.SUM, group=group)
+        cap_local, total = int(t[0]), int(t[1])
+        ent = _FUSED[key] = (cap_local, comm, FusedDistPlan(spec, comm, cap_local, max(total, cap_local * P),
+                                                            vals is not None, group))
+    k, v, _, w0 = ent[2].run(keys, vals)
+    return k, v, w0
 
 
 # ---------------------------------------------------------------------------

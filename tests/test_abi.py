@@ -223,6 +223,13 @@ def test_dist_run_argument_errors_without_gpu():
     assert L.ms_plan_workspace_size(h, 4096, ctypes.byref(ws)) == _abi.MS_OK
     assert b.value >= ws.value + 4096 * 4 + 4 * 8 * 8                             # staging + counts
     assert L.ms_dist_workspace_size(h, 4096, 0, ctypes.byref(b)) == _abi.MS_ERR_INVALID_ARG
+    wins = (ctypes.c_void_p * 1)(B)
+    assert L.ms_dist_run_fused(h, None, A, None, 100, wins, None, 100, None, None, None, W, 1 << 20, None) == \
+        _abi.MS_ERR_INVALID_ARG                                                   # no communicator
+    assert L.ms_dist_run_fused(h, P(0x40000000), A, A, 100, wins, wins, 100, None, None, None, W, 1 << 20,
+                               None) == _abi.MS_ERR_UNSUPPORTED                   # values on a key-only plan
+    assert L.ms_dist_workspace_size_fused(h, 4096, 9, ctypes.byref(b)) == _abi.MS_ERR_INVALID_ARG  # > 8 ranks
+    assert L.ms_dist_workspace_size_fused(h, 4096, 4, ctypes.byref(b)) == _abi.MS_OK
     cm = ctypes.c_void_p()
     assert L.ms_nccl_comm_init(ctypes.byref(cm), 2, 2, A, 0) == _abi.MS_ERR_INVALID_ARG   # rank >= nranks
     assert L.ms_nccl_comm_init(None, 2, 0, A, 0) == _abi.MS_ERR_INVALID_ARG

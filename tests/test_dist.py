@@ -256,3 +256,34 @@ def test_dist_run_nccl_single_rank(kind, m, kv):
         if kv:
             assert np.array_equal(wv.cpu().numpy().view(np.uint32), evo)
     comm.close()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("kind,m,kv", [("delta", 8, False), ("splitters", 32, True), ("delta", 5, True)])
+def test_dist_run_fused_single_rank(kind, m, kv):
+    """ms_dist_run_fused (local K1 + K2, NCCL count all-gather, targets, the scatter post-scan into
+    the window, NCCL barrier) on a one-rank communicator with an explicit window: bit-exact vs the
+    oracle, offsets_global included, repeated runs."""
+    from paper_conf_ppopp_ashkianidmo16_b200.dist import FusedDistPlan, NcclComm
+    torch.cuda.set_device(0)
+    spec, ospec, ranges = _case(kind, m)
+    n = (1 << 22) + 333
+    keys = W.keys_np(n, 6, "hot", m, ranges)
+    vals = W.values_np(n, 6, "index") if kv else None
+    comm = NcclComm.single(0)
+    wk = torch.empty(n + 1, dtype=torch.int32, device="cuda")
+    wv = torch.empty(n + 1, dtype=torch.int32, device="cuda") if kv else None
+    fp = FusedDistPlan(spec, comm, n, n, with_values=kv,
+                       peer_windows=([wk.data_ptr()], [wv.data_ptr()] if kv else None))
+    kd = torch.from_numpy(keys.view(np.int32).copy()).cuda()
+    vd = torch.from_numpy(vals.view(np.int32).copy()).cuda() if kv else None
+    eko, evo, eoff = oracle.multisplit(ospec, keys, vals)
+    for _ in range(2):
+        wk.fill_(-1)
+        _, _, offg, ws = fp.run(kd, vd)
+        torch.cuda.synchronize()
+        assert ws == 0 and np.array_equal(offg, eoff)
+        assert np.array_equal(wk[:n].cpu().numpy().view(np.uint32), eko)
+        if kv:
+            assert np.array_equal(wv[:n].cpu().numpy().view(np.uint32), evo)
+    comm.close()
