@@ -57,15 +57,15 @@ struct K3vLayout {
   static constexpr int CNTB = MP * RS;
   // byte offsets from the 1024-byte-aligned base (128B swizzle needs 1024 B alignment)
   static constexpr int O_SK = 0;                          // [STAGES][T] staged keys
-  static constexpr int O_SV = O_SK + STAGES * TB;         // [1][T] staged values (key-value)
-  static constexpr int O_KS = O_SV + (KV ? TB : 0);       // reordered keys
+  static constexpr int O_SV = O_SK + STAGES * TB;         // [STAGES][T] staged values
+  static constexpr int O_KS = O_SV + (KV ? STAGES * TB : 0);  // reordered keys
   static constexpr int O_VS = O_KS + KSR * 4;             // reordered values
   static constexpr int O_CNT = O_VS + (KV ? KSR * 4 : 0); // counters
   static constexpr int O_META = O_CNT + CNTB;             // [2][MW] words (tile parity)
   static constexpr int O_WS = O_META + 2 * MW * 4;        // warp sums [16]
   static constexpr int O_TOT = O_WS + 16 * 4;             // ONE: this range's bucket totals [32]
-  static constexpr int O_BAR = (O_TOT + 32 * 4 + 7) & ~7; // mbarriers: keys [STAGES], values [1]
-  static constexpr int O_SPL = O_BAR + (STAGES + 1) * 8;  // SPLITTERS: padded splitters [256] + bin table
+  static constexpr int O_BAR = (O_TOT + 32 * 4 + 7) & ~7; // mbarriers: keys [STAGES], values [STAGES]
+  static constexpr int O_SPL = O_BAR + 2 * STAGES * 8;    // SPLITTERS: padded splitters [256] + bin table
   static constexpr int O_TBL = O_SPL + kMaxM * 4;
   static constexpr int BYTES = O_SPL;                     // + 1024 alignment slack at launch
   static constexpr int BYTES_SPL = O_TBL + kSplBins * 4;
@@ -201,7 +201,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   auto issue = [&](uint32_t it, bool values) {  // one thread: TMA of sequence `it` into its stage
     const uint64_t tile = seq_tile(it, values);
     if (tile >= Lfull) return;
-    const int st = values ? 0 : (int)(it % STAGES);  // values: one stage (refilled after the scatter)
+    const int st = (int)(it % STAGES);
     if (!values) {
       mbar_arrive_expect_tx(bar_k + st, TB);
       tma_load_2d(sm + Ly::O_SK + st * TB, &tmk, 0, (int)(tile * (T / 32)), bar_k + st);
@@ -213,14 +213,16 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 
   if (tid == 0) {
 #pragma unroll
-    for (int s = 0; s < STAGES; ++s) mbar_init(bar_k + s, 1);
-    mbar_init(bar_v, 1);
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(bar_k + s, 1);
+      mbar_init(bar_v + s, 1);
+    }
     fence_mbar_init();
     const uint32_t nk = ONE ? (P1TMA ? 2 * nf : nf) : iters, nv = ONE ? nf : iters;
     for (uint32_t s = 0; s < (uint32_t)STAGES; ++s) {
       if (s < nk) issue(s, false);
       if constexpr (KV) {
-        if (s == 0 && s < nv) issue(0, true);
+        if (s < nv) issue(s, true);
       }
     }
   }
@@ -377,8 +379,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     const uint32_t kq = ONE ? (P1TMA ? nf : 0u) + it - ptail : it, vq = ONE ? it - ptail : it;
     const int st = (int)(kq % STAGES);
     const uint32_t ph = (kq / STAGES) & 1u;
-    const int vst = 0;
-    const uint32_t vph = vq & 1u;
+    const int vst = (int)(vq % STAGES);
+    const uint32_t vph = (vq / STAGES) & 1u;
     uint32_t *meta = reinterpret_cast<uint32_t *>(sm + Ly::O_META) + (it & 1) * Ly::MW;
     uint32_t *rowS = meta;          // [MP+4]
     uint32_t *Pj = meta + MP + 4;   // [MP]
@@ -611,7 +613,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA (async proxy)
     __syncthreads();
     if constexpr (KV) {  // the value stage is free again: refill it
-      if (FULL && tid == 0 && vq + 1 < (ONE ? nf : iters)) issue(vq + 1, true);
+      if (FULL && tid == 0 && vq + STAGES < (ONE ? nf : iters)) issue(vq + STAGES, true);
     }
 
     // ---- 4. bucket runs: SPB threads per bucket share its <= 3 head keys,
@@ -795,8 +797,7 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
 template <int KIND, bool KV, int LOGMP, int IDB>
 inline cudaError_t k3v_launch_n(const K3pArgs &a) {
   constexpr int NT = 256;
-  // key stages (values: one): key-value 2 (two CTAs of ~104-109 KB per SM), key-only m <= 8: 3 (still 3 CTAs/SM)
-  constexpr int STAGES = KV ? 2 : (LOGMP <= 3 ? 3 : 2);
+  constexpr int STAGES = KV ? 1 : (LOGMP <= 3 ? 3 : 2);  // m <= 8 key-only: 3 stages still fit 3 CTAs/SM
   if (a.nt != 256) {  // ablation (NW sweep): 2 or 4 warps per CTA, ranged variant, one bucket kind
     if constexpr (KIND == SHIFT) {
       if (a.ranged != 1) return cudaErrorNotSupported;
