@@ -488,3 +488,75 @@ def test_parity_nw_ablation(variant, m):
             got = _run_case(case, variant)
             assert got[3].geometry(n)[0] == T
             _assert_equal(case, got, _expect(case), f"{variant} m={m} n={n} kv={kv}")
+
+
+# ---------------------------------------------------------------- the largest sizes (n up to 2^32 - 5)
+def _torch_ids(keys_i32, kind, m, spl=None, delta=None):
+    k = keys_i32.to(torch.int64) & 0xFFFFFFFF
+    if kind == "delta":
+        return torch.clamp(k // delta, max=m - 1)
+    return torch.searchsorted(torch.as_tensor(spl.astype(np.int64), device=keys_i32.device), k, side="left")
+
+
+def test_max_size_kv_vs_definition():
+    """n = 2^31 + 7 key-value pairs (C5's total on one GPU, m = 32 splitters), the whole output
+    element for element against the definition evaluated independently with torch on the GPU:
+    bucket j of the output must be exactly the input's elements with id j, in input order
+    (Eq. (1)) -- built chunk by chunk with boolean selection (torch's sort stops at
+    2^31 elements) -- and the offsets the exclusive scan of the id histogram."""
+    P = _pkg()
+    n, m = (1 << 31) + 7, 32
+    spl = W.gen_splitters(m, W.SEEDS["C5"])
+    keys = W.keys_torch(n, W.SEEDS["C5"], "cuda")
+    vals = W.values_torch(n, W.SEEDS["C5"], "cuda", "random")
+    plan = P.Plan(P.BucketSpec.from_splitters(spl.tolist()), n, with_values=True)
+    ko, vo, off = plan.run(keys, vals)
+    torch.cuda.synchronize()
+    assert plan.last_launches() == 3 - (plan.geometry(n)[2])  # ranged (2) at this size
+    ids = _torch_ids(keys, "splitters", m, spl=spl).to(torch.uint8)
+    hist = torch.bincount(ids, minlength=m).to(torch.int64)
+    exp_off = torch.cat([torch.zeros(1, dtype=torch.int64, device="cuda"), torch.cumsum(hist, 0)])
+    assert torch.equal(off.to(torch.int64) & 0xFFFFFFFF, exp_off)
+    cursor = exp_off[:-1].clone()
+    C = 1 << 28
+    for c in range(0, n, C):
+        idc, kc, vc = ids[c:c + C], keys[c:c + C], vals[c:c + C]
+        for j in range(m):
+            sel = idc == j
+            ek, ev = kc[sel], vc[sel]
+            a = int(cursor[j])
+            assert torch.equal(ko[a:a + ek.numel()], ek), f"keys of bucket {j}, input chunk {c}"
+            assert torch.equal(vo[a:a + ev.numel()], ev), f"values of bucket {j}, input chunk {c}"
+            cursor[j] += ek.numel()
+    assert torch.equal(cursor, exp_off[1:])
+
+
+def test_max_size_ko_properties():
+    """n = 2^32 - 5 keys (the largest n the ABI takes), key-only, m = 8 delta (one ONE launch): the
+    output is the same multiset as the input (order-insensitive 64-bit hashes), its bucket ids never
+    decrease, and the offsets are exactly the id boundaries (for key-only output, equal keys are
+    interchangeable, so these properties determine the result)."""
+    P = _pkg()
+    n, m, delta = (1 << 32) - 5, 8, 1 << 29
+    keys = W.keys_torch(n, 424242, "cuda")
+    plan = P.Plan(P.BucketSpec.delta_range(m, delta), n)
+    ko, _, off = plan.run(keys)
+    torch.cuda.synchronize()
+    assert plan.last_launches() == 1
+
+    def mh(t):  # order-insensitive multiset hash of u32 values: sum of a mixing function, mod 2^64
+        h = 0
+        for c in range(0, t.numel(), 1 << 28):
+            x = t[c:c + (1 << 28)].to(torch.int64) & 0xFFFFFFFF
+            x = (x ^ (x >> 16)) * 0x45D9F3B
+            x = (x ^ (x >> 13)) * 0x2C1B3C6D
+            h = (h + int(x.sum())) & ((1 << 64) - 1)
+        return h
+    assert mh(ko) == mh(keys)
+    offh = (off.to(torch.int64) & 0xFFFFFFFF).tolist()
+    assert offh[0] == 0 and offh[m] == n and all(a <= b for a, b in zip(offh, offh[1:]))
+    for j in range(m):  # every position in [off[j], off[j+1]) has id j (checked chunk-wise)
+        for c in range(offh[j], offh[j + 1], 1 << 28):
+            seg = ko[c:min(c + (1 << 28), offh[j + 1])]
+            ids = _torch_ids(seg, "delta", m, delta=delta)
+            assert bool((ids == j).all()), f"bucket {j} chunk at {c}"
