@@ -556,6 +556,8 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparato
         "gpu_launches": launches * K, "launches_per_step": launches, "tile": T, "tiles": L,
         "variant": ["tile", "ranged", "one", "two-pass"][variant], "clocks": clocks.result(),
     }
+    if n <= (1 << 22) and world == 1:  # launch-bound sizes: also the CUDA-graph replay rate
+        res["graph_replay"] = measure_graph(cfg, plan, keys, vals, ids)
     if comparators:
         comp = measure_comparators(cfg, plan, keys, vals, ids, 3, flush)
         for v in comp.values():
@@ -568,6 +570,38 @@ def bench_config(name, cfg, K, Wm, device, world, rank, with_e2e=True, comparato
     del keys, vals, ids, flush
     torch.cuda.empty_cache()
     return res
+
+
+def measure_graph(cfg, plan, keys, vals, ids, calls=20, reps=10):
+    """Small, launch-bound workloads: `calls` back-to-back ms_run calls captured in
+    one CUDA graph and replayed (L2-warm: the inputs stay resident between calls) -- the per-call
+    device time without per-call launch gaps."""
+    import torch
+    ko = torch.empty_like(keys)
+    vo = torch.empty_like(vals) if vals is not None else None
+    off = torch.empty(cfg["m"] + 1, dtype=torch.int32, device=keys.device)
+    ws = plan.workspace(keys.numel())
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            plan.run(keys, vals, ids, keys_out=ko, vals_out=vo, offsets=off, workspace=ws)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(calls):
+            plan.run(keys, vals, ids, keys_out=ko, vals_out=vo, offsets=off, workspace=ws)
+    g.replay()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        g.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    us = e0.elapsed_time(e1) * 1e3 / (reps * calls)
+    return {"per_call_us": round(us, 3), "value": round(keys.numel() / (us * 1e-6) / 1e9, 2), "unit": "G keys/s",
+            "note": f"{calls} back-to-back ms_run calls captured in one CUDA graph, replayed {reps}x; L2-warm"}
 
 
 NVLINK_GBS_PER_DIR = 900.0  # NVLink 5 per GPU per direction (NVSwitch: uniform to every peer)
@@ -752,6 +786,8 @@ def run_ours(args, name, cfg, world, rank, local):
                              "k1_frac": r["roofline"]["k1_prescan_frac"],
                              "stages_ms": {k: round(v, 4) for k, v in r["stages_ms"].items()},
                              "comparators": r.get("comparators"), "clocks": r["clocks"]}
+                if "graph_replay" in r:
+                    extra[nm]["graph_replay"] = r["graph_replay"]
                 log(f"extra {nm}: {r['value']:.1f} G keys/s frac {r['whole_step_frac']:.3f}")
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:

@@ -560,3 +560,33 @@ def test_max_size_ko_properties():
             seg = ko[c:min(c + (1 << 28), offh[j + 1])]
             ids = _torch_ids(seg, "delta", m, delta=delta)
             assert bool((ids == j).all()), f"bucket {j} chunk at {c}"
+
+
+@pytest.mark.parametrize("kind,m,kv,n", [("lowbits", 2, False, 1 << 20), ("splitters", 32, True, 100003),
+                                         ("delta", 256, False, 50000), ("delta", 1000, True, 70001)])
+def test_cuda_graph_capture(kind, m, kv, n):
+    """ms_run is stream-ordered with no host synchronisation, so it can be captured in a CUDA graph
+    (ONE's cooperative launch, the 3-kernel path and the two-pass plan alike) and replayed: the
+    replayed output equals the oracle's."""
+    P = _pkg()
+    if m > 256:
+        case = _wide_case(kind, m, dict(delta=4000037), n, seed=5, kv=kv)
+    else:
+        case = make_case(kind, m, n, seed=5, kv=kv)
+    plan = P.Plan(P.BucketSpec(**case["spec_kw"]), n, with_values=kv)
+    kd, vd = to_dev(case["keys"]), to_dev(case["vals"])
+    ko, vo = torch.empty_like(kd), (torch.empty_like(vd) if kv else None)
+    off = torch.empty(m + 1, dtype=torch.int32, device="cuda")
+    ws = plan.workspace(n)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        plan.run(kd, vd, keys_out=ko, vals_out=vo, offsets=off, workspace=ws)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        plan.run(kd, vd, keys_out=ko, vals_out=vo, offsets=off, workspace=ws)
+    ko.fill_(0)
+    g.replay()
+    torch.cuda.synchronize()
+    _assert_equal(case, (from_dev(ko), from_dev(vo), from_dev(off), plan), _expect(case), f"graph {kind} m={m}")
