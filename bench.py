@@ -813,7 +813,7 @@ def run_ours(args, name, cfg, world, rank, local):
             "tile": res["tile"], "variant": res["variant"], "launches_per_step": res["launches_per_step"],
             "extra": extra,
         }
-        for k in ("comparators", "local_step", "bounds"):
+        for k in ("comparators", "local_step", "bounds", "graph_replay"):
             if k in res:
                 out[k] = res[k]
         print(json.dumps(out), flush=True)
