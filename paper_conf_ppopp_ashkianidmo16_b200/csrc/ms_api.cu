@@ -175,7 +175,7 @@ cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *key
                                              flag);                                                \
   }
   if (p->spec.m > 32) {  // one warp per tile, lane-private byte counters (k1w_prescan)
-    const size_t smw = (kMaxM + (size_t)kWarps * ((p->spec.m + 3) / 4) * 32) * 4;
+    const size_t smw = (kMaxM + (size_t)kWarps * (kMaxM / 4) * 32) * 4;
     const unsigned grid = (unsigned)((g.L + kWarps - 1) / kWarps);
     if (g.R == 8) {
       set_smem(k1w_prescan<KIND, 64>, smw);

@@ -244,7 +244,7 @@ k1w_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   uint32_t *spl_s = smem;                                        // kMaxM words (SPLITTERS)
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t m = p.m, groups = (m + 3) >> 2;                  // row groups of 4 buckets
-  uint32_t *cw = smem + kMaxM + warp * groups * 32;               // this warp's [groups][32] words
+  uint32_t *cw = smem + kMaxM + warp * (kMaxM / 4) * 32;          // this warp's [groups][32] words
   uint8_t *mine = reinterpret_cast<uint8_t *>(cw + lane);         // byte (j & 3) at + (j >> 2) * 128
   const uint64_t tile = (uint64_t)blockIdx.x * kWarps + warp;
   const uint64_t base = tile * T;
@@ -269,29 +269,9 @@ k1w_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
     uint8_t *a = mine + (id >> 2) * 128 + (id & 3);
     *a = (uint8_t)(*a + 1);
   };
-  if (nt == T && KIND != IDS) {
-    // 16 keys per lane per step (4 x 512-byte spans); the next step's loads are issued before this
-    // step is counted (register double buffer), so every warp keeps 4 KB of loads in flight
-    uint4 va[4], vb[4];
-    auto ld = [&](uint32_t s, uint4 *v) {
-#pragma unroll
-      for (int c = 0; c < 4; ++c) v[c] = __ldg(reinterpret_cast<const uint4 *>(keys + base + (uint64_t)s * 512) + c * 32 + lane);
-    };
-    auto cnt = [&](const uint4 *v) {
-#pragma unroll
-      for (int c = 0; c < 4; ++c) { count(v[c].x); count(v[c].y); count(v[c].z); count(v[c].w); }
-    };
-    ld(0, va);
-#pragma unroll 1
-    for (uint32_t s = 0; s < (uint32_t)KPT / 16; s += 2) {
-      ld(s + 1, vb);
-      cnt(va);
-      if (s + 2 < (uint32_t)KPT / 16) ld(s + 2, va);
-      cnt(vb);
-    }
-  } else if (nt == T) {
+  if (nt == T) {
 #pragma unroll 2
-    for (uint32_t s = 0; s < (uint32_t)KPT / 16; ++s) {  // 16 ids per lane per step
+    for (uint32_t s = 0; s < (uint32_t)KPT / 16; ++s) {  // 16 keys per lane per step: 4 x 512-byte spans
       const uint64_t sb = base + (uint64_t)s * 512;
       if constexpr (KIND == IDS) {
         if (p.id_bytes == 1) {  // 16 ids per lane: one 16-byte load, lanes contiguous
