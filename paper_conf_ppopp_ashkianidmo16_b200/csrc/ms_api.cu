@@ -174,20 +174,6 @@ cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *key
     k<<<(unsigned)grid, kThreads, smem, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, zero_words, \
                                              flag);                                                \
   }
-  if (p->spec.m > 32) {  // one warp per tile, lane-private byte counters (k1w_prescan)
-    const size_t smw = (kMaxM + (size_t)kWarps * (kMaxM / 4) * 32) * 4;
-    const unsigned grid = (unsigned)((g.L + kWarps - 1) / kWarps);
-    if (g.R == 8) {
-      set_smem(k1w_prescan<KIND, 64>, smw);
-      k1w_prescan<KIND, 64><<<grid, kThreads, smw, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr, zero_words,
-                                                        flag);
-    } else {
-      set_smem(k1w_prescan<KIND, 128>, smw);
-      k1w_prescan<KIND, 128><<<grid, kThreads, smw, s>>>(keys, ids, n, (uint32_t)g.L, H, p->bp, zero_ptr,
-                                                         zero_words, flag);
-    }
-    return cudaGetLastError();
-  }
   switch (g.R) {  // 16 keys per thread; T = 2048 tiles are counted two per CTA
     case 8: MS_K1(16, 2) break;
     case 16: MS_K1(16, 1) break;

@@ -224,110 +224,6 @@ k1a_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   }
 }
 
-// K1 for 32 < m <= 256, one WARP per tile (T = 32 * KPT keys; a CTA = 8 warps = 8 tiles): each
-// lane counts its KPT keys (read as coalesced 512-byte warp spans) into lane-PRIVATE byte
-// counters -- bucket j of lane l at byte (j & 3) of word l of row group j >> 2, so the 32 lanes
-// always hit 32 different banks and no atomics are needed (at most KPT <= 255 per byte) -- then
-// lane l sums row groups l and l + 32 over the 32 lanes' words (rotated word order:
-// conflict-free; even/odd bytes in 16-bit halves) and writes those 4-bucket columns of H.  The
-// per-warp counter block is ceil(m/4) * 128 bytes (8 KB at m = 256) and is reduced once per tile:
-// ~2 B of shared-memory reads per key, against one shared atomic per key (and its MIO-queue
-// throttling, ncu: mio_throttle 22.6 per issued instruction at m = 256) in k1a_prescan.
-template <int KIND, int KPT>
-__global__ void __launch_bounds__(kThreads)
-k1w_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
-            uint32_t L, uint32_t *__restrict__ H, const __grid_constant__ BucketParams p,
-            uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
-  constexpr int T = 32 * KPT;  // keys per tile (= per warp)
-  static_assert(KPT <= 255 && KPT % 16 == 0, "byte counters, 16-key steps");
-  extern __shared__ __align__(16) uint32_t smem[];
-  uint32_t *spl_s = smem;                                        // kMaxM words (SPLITTERS)
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t m = p.m, groups = (m + 3) >> 2;                  // row groups of 4 buckets
-  uint32_t *cw = smem + kMaxM + warp * (kMaxM / 4) * 32;          // this warp's [groups][32] words
-  uint8_t *mine = reinterpret_cast<uint8_t *>(cw + lane);         // byte (j & 3) at + (j >> 2) * 128
-  const uint64_t tile = (uint64_t)blockIdx.x * kWarps + warp;
-  const uint64_t base = tile * T;
-  const uint32_t nt = tile < L ? (uint32_t)umin64(T, n - base) : 0u;
-  pdl_trigger();
-  for (uint32_t i = blockIdx.x * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
-  if constexpr (KIND == SPLITTERS) {
-    for (uint32_t i = tid; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
-    __syncthreads();
-  }
-  for (uint32_t g = 0; g < groups; ++g) cw[g * 32 + lane] = 0u;
-  __syncwarp();
-  uint32_t bad = 0;
-  auto count = [&](uint32_t raw) {
-    uint32_t id;
-    if constexpr (KIND == IDS) {
-      bad |= raw > p.mmask;
-      id = min(raw, p.mmask);
-    } else {
-      id = bucket_of_key<KIND>(raw, p, spl_s);
-    }
-    uint8_t *a = mine + (id >> 2) * 128 + (id & 3);
-    *a = (uint8_t)(*a + 1);
-  };
-  if (nt == T) {
-#pragma unroll 2
-    for (uint32_t s = 0; s < (uint32_t)KPT / 16; ++s) {  // 16 keys per lane per step: 4 x 512-byte spans
-      const uint64_t sb = base + (uint64_t)s * 512;
-      if constexpr (KIND == IDS) {
-        if (p.id_bytes == 1) {  // 16 ids per lane: one 16-byte load, lanes contiguous
-          const uint4 w = __ldg(reinterpret_cast<const uint4 *>((const uint8_t *)ids + sb) + lane);
-          const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
-#pragma unroll
-          for (int q = 0; q < 16; ++q) count((ww[q >> 2] >> (8 * (q & 3))) & 255u);
-        } else {
-          uint4 v[4];
-#pragma unroll
-          for (int c = 0; c < 4; ++c) v[c] = __ldg(reinterpret_cast<const uint4 *>((const uint32_t *)ids + sb) + c * 32 + lane);
-#pragma unroll
-          for (int c = 0; c < 4; ++c) { count(v[c].x); count(v[c].y); count(v[c].z); count(v[c].w); }
-        }
-      } else {
-        uint4 v[4];
-#pragma unroll
-        for (int c = 0; c < 4; ++c) v[c] = __ldg(reinterpret_cast<const uint4 *>(keys + sb) + c * 32 + lane);
-#pragma unroll
-        for (int c = 0; c < 4; ++c) { count(v[c].x); count(v[c].y); count(v[c].z); count(v[c].w); }
-      }
-    }
-  } else {
-    for (uint32_t i = lane; i < nt; i += 32) {
-      if constexpr (KIND == IDS)
-        count(p.id_bytes == 1 ? (uint32_t)((const uint8_t *)ids)[base + i] : ((const uint32_t *)ids)[base + i]);
-      else
-        count(keys[base + i]);
-    }
-  }
-  if constexpr (KIND == IDS) {
-    if (p.validate && __any_sync(0xFFFFFFFFu, bad) && lane == 0) atomicOr(err_flag, 1u);
-  }
-  __syncwarp();
-  if (nt == 0) return;
-  // column of H: lane l sums row groups l and l + 32 over the 32 lanes' words
-#pragma unroll
-  for (uint32_t gg = 0; gg < 2; ++gg) {
-    const uint32_t g = lane + 32 * gg;
-    if (g < groups) {
-      uint32_t ev = 0, od = 0;  // bytes 0,2 / 1,3 of the 32 words, in 16-bit halves
-#pragma unroll 8
-      for (uint32_t k = 0; k < 32; ++k) {
-        const uint32_t w = cw[g * 32 + ((k + lane) & 31)];
-        ev += w & 0x00FF00FFu;
-        od += (w >> 8) & 0x00FF00FFu;
-      }
-      const uint32_t j0 = 4 * g;
-      const uint32_t c[4] = {ev & 0xFFFFu, od & 0xFFFFu, ev >> 16, od >> 16};
-#pragma unroll
-      for (uint32_t e = 0; e < 4; ++e)
-        if (j0 + e < m) H[(uint64_t)(j0 + e) * L + tile] = c[e];
-    }
-  }
-}
-
 // Persistent form of K1 for MS_SPLITTERS: the bin table (ms_device.cuh) is
 // built once per CTA, then the CTA walks tile groups with a stride of gridDim.x.
 template <int KIND, int KPT, int SUBT>
