@@ -217,6 +217,19 @@ __device__ __forceinline__ void sts_u16(uint32_t a, uint32_t v) {
 __device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
   asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
+// u16 counter at shared address a (2-byte aligned) incremented by a 32-bit shared atomic on its
+// word (the other half belongs to another thread and never carries: counts stay < 2^16); returns
+// the counter's old value.  No load -> add -> store round trip in the issuing thread, so
+// consecutive increments pipeline.
+__device__ __forceinline__ uint32_t atom_inc_u16(uint32_t a) {
+  const uint32_t sh = (a & 2u) * 8u;
+  uint32_t old;
+  asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(a & ~3u), "r"(1u << sh) : "memory");
+  return (old >> sh) & 0xFFFFu;
+}
+__device__ __forceinline__ void red_inc_u16(uint32_t a) {  // the same, old value not needed
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a & ~3u), "r"(1u << ((a & 2u) * 8u)) : "memory");
+}
 
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 inline uint64_t umin64_host(uint64_t a, uint64_t b) { return a < b ? a : b; }

@@ -268,7 +268,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     __syncthreads();
     auto count_id = [&](uint32_t id) {
       const uint32_t a = ccol + id * RS;
-      sts_u16(a, lds_u16(a) + 1);
+      red_inc_u16(a);
     };
     auto count1 = [&](uint32_t key) { count_id(id_of(key)); };
     // counting needs no key-to-thread order: coalesced 128-bit loads (chunk j*NT + tid of the
@@ -448,8 +448,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
           if constexpr (KIND == IDS) id = __byte_perm(idk[c], 0u, 0x4440u + j);
           else id = id_of(kk[j]);
           const uint32_t a = ccol + id * RS;
-          const uint32_t r = lds_u16(a);
-          sts_u16(a, r + 1);
+          const uint32_t r = atom_inc_u16(a);
           rk[c] |= r << (8 * j);
           if constexpr (KEEP_ID && KIND != IDS) idk[c] |= id << (8 * j);
         }
