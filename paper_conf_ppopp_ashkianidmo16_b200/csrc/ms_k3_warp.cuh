@@ -87,13 +87,11 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
       peers = ~diff;
     }
     const uint32_t rank = __popc(peers & lt);
-    // the highest lane of each group advances the warp's counter of its bucket with one shared
-    // atomic and hands the old value to its group (the shuffle also orders this round's atomics
-    // before the next round's)
-    const uint32_t leader = 31u - __clz(peers);
-    uint32_t old = 0;
-    if (valid && lane == leader) old = atomicAdd(cnt_w + id, (uint32_t)__popc(peers));
-    const uint32_t before = __shfl_sync(0xFFFFFFFFu, old, leader);
+    uint32_t before = 0;
+    if (valid) before = cnt_w[id];
+    __syncwarp();
+    if (valid && (peers & gt) == 0) cnt_w[id] = before + __popc(peers);
+    __syncwarp();
     kreg[r] = key;
     if constexpr (KV) vreg[r] = vals_s[pos];
     pk[r] = ((before + rank) << 8) | (id & 255u);
