@@ -767,7 +767,9 @@ template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ON
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
   constexpr int KPT = 16;
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
-  constexpr int MINB = (KV ? 2 : 3) * (256 / NT);
+  // CTAs per SM the register budget is sized for: key-value 2, key-only 3 -- and 4 for the
+  // two-stage key-only m <= 8 form used on smaller inputs (k3v_launch_n)
+  constexpr int MINB = (KV ? 2 : (STAGES == 2 && LOGMP <= 3 ? 4 : 3)) * (256 / NT);
   auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE, DIRECT, IDB>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -805,7 +807,15 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
     }
     return cudaErrorNotSupported;
   }
-  if (a.ranged == 2) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true, false, IDB>(a);
+  if (a.ranged == 2) {
+    // ONE, key-only, m <= 8: up to 64 tiles per SM two key stages at 4 CTAs/SM (more CTAs to share
+    // the fixed cost and the tail: C2, n = 2^25, 408 -> 418 G keys/s), above that three stages at
+    // 3 CTAs/SM (the deeper prefetch wins for long streams: m8 KO at 2^28 518 vs 499)
+    if constexpr (!KV && LOGMP <= 3) {
+      if (a.L <= 64ull * (uint64_t)a.sms) return k3v_launch_one<KIND, KV, LOGMP, NT, 2, true, true, false, IDB>(a);
+    }
+    return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true, false, IDB>(a);
+  }
   if (a.direct) {  // ablation: instantiated for the one-shift bucket kind only (SHIFT: DELTA with m*delta = 2^32)
     if constexpr (KIND == SHIFT) return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, true>(a);
     return cudaErrorNotSupported;
