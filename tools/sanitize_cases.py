@@ -24,8 +24,8 @@ n = int(sys.argv[1]) if len(sys.argv) > 1 else 3 * 4096 * 148 + 77  # > 1 tile p
 cases = [("delta", 8, False, "one"), ("delta", 8, True, "one"), ("splitters", 32, False, "one"),
          ("ids", 32, True, "one"), ("lowbits", 16, True, "ranged"), ("splitters", 32, True, "ranged"),
          ("delta", 32, False, "3k"), ("ids", 5, True, "3k"), ("delta", 256, False, "3k"),
-         ("splitters", 200, True, "3k"), ("ids", 100, False, "3k"), ("delta", 256, True, "ranged"),
-         ("splitters", 100, False, "ranged")]
+         ("splitters", 200, True, "3k"), ("ids", 100, False, "3k"), ("delta", 256, True, None),
+         ("splitters", 100, False, None), ("delta", 8, False, "nw2"), ("delta", 32, True, "nw4")]
 fails = 0
 for kind, m, kv, variant in cases:
     case = make_case(kind, m, n, seed=m + 3, kv=kv, dist="binomial")
