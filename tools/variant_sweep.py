@@ -1,6 +1,6 @@
 """Which variant wins where (the measured rule of ms_api.cu choose_variant):
 G keys/s of ONE / ranged / tile for a set of workloads at several n.
-usage: python tools/variant_sweep.py [steps] > profiles/r02_variants.md"""
+usage: python tools/variant_sweep.py [steps] [base,base,...] > profiles/r02_variants.md"""
 import os
 import sys
 
@@ -12,8 +12,9 @@ import bench  # noqa: E402
 steps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
 print("| workload | n | one | ranged | tile | default (variant) |")
 print("|---|---|---|---|---|---|")
-for base in ("C3", "C3bin", "sweep_m2_kv", "sweep_m8_kv", "sweep_m16_kv", "sweep_m32_kv", "IDSkv", "sweep_m32_ko",
-             "sweep_m8_ko"):
+BASES = ("C3", "C3bin", "sweep_m2_kv", "sweep_m8_kv", "sweep_m16_kv", "sweep_m32_kv", "IDSkv", "sweep_m32_ko",
+         "sweep_m8_ko", "sweep_m64_kv", "sweep_m64_ko")
+for base in (sys.argv[2].split(",") if len(sys.argv) > 2 else BASES):
     for e in (23, 25, 26, 27):
         cfg = dict(bench.CONFIGS[base], n=1 << e)
         row = []
