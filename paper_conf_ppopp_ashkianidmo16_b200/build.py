@@ -20,7 +20,8 @@ SOURCES = ["ms_api.cu", "ms_dist.cu", "ms_wide.cu", "k3_lowbits.cu", "k3_shiftc.
 HEADERS = ["ms_k3_v2.cuh", "ms_kernels.cuh", "ms_device.cuh", "ms_k3_warp.cuh", "ms_k3p_args.h", "ms_ranged.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr"]
+FLAGS = ["-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
+         *os.environ.get("MS_NVCC_EXTRA", "").split()]  # (experiments: extra -D flags)
 
 
 def _deps_mtime() -> float:

@@ -388,13 +388,16 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     uint32_t *Dj = Gj + MP;         // [MP] DIRECT: G_j - P_j
 
     // ---- 0. zero the counters (last read by the previous tile's scatter,
-    // before its final barrier); publish this tile's G column
+    // before its final barrier) -- the plain 16-byte chunks only, not the
+    // padding (chunk c of row r at r * RS + 16 * (c + c / 8)); publish this
+    // tile's G column
     {
-      uint4 *c4 = reinterpret_cast<uint4 *>(cnt);
+      constexpr int CPR = 2 * NT / 16, PCH = MP * CPR;
 #pragma unroll
-      for (int i = 0; i < (Ly::CNTB / 16 + NT - 1) / NT; ++i) {
+      for (int i = 0; i < (PCH + NT - 1) / NT; ++i) {
         const int idx = i * NT + tid;
-        if (idx < Ly::CNTB / 16) c4[idx] = make_uint4(0, 0, 0, 0);
+        const int r = idx / CPR, c = idx % CPR;
+        if (idx < PCH) *reinterpret_cast<uint4 *>(cnt + r * RS + 16 * (c + (c >> 3))) = make_uint4(0, 0, 0, 0);
       }
     }
     if constexpr (!RANGED) {
