@@ -134,7 +134,9 @@ ms_status ms_plan_workspace_size(ms_plan_t plan, uint64_t n, size_t *bytes);
 /* Tile geometry the plan uses for n elements: tile = T (keys per subproblem),
  * num_tiles = L = ceil(n / T), variant = 0 (tile, 3 launches), 1 (ranged, 2)
  * or 2 (ONE, 1) -- the variant a run of n elements (key-value if the plan has
- * values) takes. */
+ * values) takes.  T and L are those of the tile variant and the stage-wise
+ * calls; a key-only ONE run with 17..32 computed-id buckets walks 8192-key
+ * tiles internally. */
 ms_status ms_plan_geometry(ms_plan_t plan, uint64_t n, uint32_t *tile, uint64_t *num_tiles,
                            int32_t *variant);
 

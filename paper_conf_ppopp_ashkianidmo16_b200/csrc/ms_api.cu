@@ -32,7 +32,7 @@ struct ms_plan_s {
   int kkind;  // kernel-level Kind (ms_device.cuh)
   int device;  // CUDA ordinal every call of this plan runs on
   int sms;     // its SM count
-  uint32_t kpt = 16;    // K3 (m <= 32): keys per thread
+  uint32_t kpt = 16;    // K3 (m <= 32): keys per thread (32 for key-only ONE runs of 17..32 buckets)
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt = 4096
   int forced = -1;      // MS_VARIANT_* flag: the variant every run uses (-1: chosen per run)
   int direct = 0;       // MS_ABLATION_DIRECT: K3 stores keys straight to global, no local reorder
@@ -103,9 +103,9 @@ struct Geometry {
   size_t off_hc;          // CTA-range / ONE variants: range counts HC[R][m], over the H/G region
 };
 
-Geometry geometry(const ms_plan_s *p, uint64_t n) {
+Geometry geometry(const ms_plan_s *p, uint64_t n, uint32_t kpt = 0) {
   Geometry g{};
-  g.R = rounds_for(p->spec.m, n, p->kpt * p->k3nt / 256);
+  g.R = rounds_for(p->spec.m, n, (kpt ? kpt : p->kpt) * p->k3nt / 256);
   g.T = 256u * g.R;
   g.L = (n + g.T - 1) / g.T;
   g.hg_words = (uint64_t)p->spec.m * g.L;
@@ -205,7 +205,7 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
                         uint32_t *grid_out = nullptr, int pdl = 0, const RangeScan *rs = nullptr,
                         const uint32_t *rowtot = nullptr) {
   K3pArgs a{keys, vals, ids, G, ko, vo, n, (uint32_t)g.L, p->spec.m, p->spec.id_bytes,
-            p->spec.m <= 32 ? p->kpt : (uint32_t)g.R, p->k3nt, &p->bp, p->sms, s};
+            p->spec.m <= 32 ? g.T / 256 : (uint32_t)g.R, p->k3nt, &p->bp, p->sms, s};
   a.ranged = ranged;
   a.grid_out = grid_out;
   a.pdl = pdl;
@@ -847,8 +847,11 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
       cudaEventRecord(ev[1], s);
       cudaEventRecord(ev[2], s);
     }
-    const cudaError_t e1 = dispatch_k3(p, g, keys_in, vals_in, ids, nullptr, keys_out, vals_out, (uint32_t)n, flag,
-                                       s, 2, nullptr, 0, &rs);
+    // key-only, 17..32 buckets (computed ids): tiles of 8192 keys, 32 per thread (DESIGN.md §7:
+    // half the counter-matrix work per key; NSko 440 -> 464 G keys/s, m <= 16 slower)
+    const bool k32 = vals_in == nullptr && p->spec.m > 16 && p->kkind != IDS && p->k3nt == 256 && !p->direct;
+    const cudaError_t e1 = dispatch_k3(p, k32 ? geometry(p, n, 32) : g, keys_in, vals_in, ids, nullptr, keys_out,
+                                       vals_out, (uint32_t)n, flag, s, 2, nullptr, 0, &rs);
     if (e1 == cudaSuccess) {
       if (ev) cudaEventRecord(ev[3], s);
       p->last_launches = 1;

@@ -243,7 +243,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   uint32_t *tot_s = reinterpret_cast<uint32_t *>(sm + Ly::O_TOT);
   if constexpr (ONE) {
     // ---- phase 1: this range's bucket counts (private u16 counter columns,
-    // folded into tot_s every 2048 tiles so that no counter exceeds 32768)
+    // folded into tot_s every 32768 / K tiles so that no counter exceeds 32768)
+    constexpr uint32_t FOLDT = 32768u / K;
     if (tid < 32) tot_s[tid] = 0;
     auto zero_cnt = [&]() {
       uint4 *c4 = reinterpret_cast<uint4 *>(cnt);
@@ -296,7 +297,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
         // RETURNED (values consumed above), not merely been issued
         __syncthreads();
         if (tid == 0 && sq + STAGES < 2 * nf) issue(sq + STAGES, false);
-        if ((sq & 2047u) == 2047u) fold();
+        if ((sq & (FOLDT - 1)) == FOLDT - 1) fold();
       }
     }
     if constexpr (KIND == IDS) {  // precomputed ids: phase 1 reads only the ids (coalesced 16-byte chunks)
@@ -313,7 +314,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
             count_id((w[q] >> 16) & 255u); count_id(w[q] >> 24);
           }
         }
-        if ((sq & 2047u) == 2047u) fold();
+        if ((sq & (FOLDT - 1)) == FOLDT - 1) fold();
       }
     }
     constexpr bool P1LD = !P1TMA && KIND != IDS;  // key-value, computed ids: plain loads of the keys
@@ -322,11 +323,11 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     for (uint32_t sq = 0; P1LD && sq < nf;) {
       if (sq + 1 < nf) ld(sq + 1, xb);
       cnt4(xa);
-      if ((sq & 2047u) == 2047u) fold();
+      if ((sq & (FOLDT - 1)) == FOLDT - 1) fold();
       if (++sq >= nf) break;
       if (sq + 1 < nf) ld(sq + 1, xa);
       cnt4(xb);
-      if ((sq & 2047u) == 2047u) fold();
+      if ((sq & (FOLDT - 1)) == FOLDT - 1) fold();
       ++sq;
     }
     if (ptail) {  // the partial last tile of the input
@@ -766,13 +767,13 @@ inline bool make_tile_map(CUtensorMap *tm, const uint32_t *ptr, uint64_t rows, u
 }
 
 template <int KIND, bool KV, int LOGMP, int NT, int STAGES, bool RANGED, bool ONE = false, bool DIRECT = false,
-          int IDB = 0>
+          int IDB = 0, int KPT = 16>
 inline cudaError_t k3v_launch_one(const K3pArgs &a) {
-  constexpr int KPT = 16;
   using Ly = K3vLayout<LOGMP, KV, NT, STAGES, KPT>;
   // CTAs per SM the register budget is sized for: key-value 2, key-only 3 -- and 4 for the
   // two-stage key-only m <= 8 form used on smaller inputs (k3v_launch_n)
-  constexpr int MINB = (KV ? 2 : (STAGES == 2 && LOGMP <= 3 ? 4 : 3)) * (256 / NT);
+  // (32 keys per thread: one key stage, 2 CTAs/SM)
+  constexpr int MINB = KPT == 32 ? 2 : (KV ? 2 : (STAGES == 2 && LOGMP <= 3 ? 4 : 3)) * (256 / NT);
   auto k = k3v_postscan<KIND, KV, LOGMP, NT, STAGES, RANGED, MINB, KPT, ONE, DIRECT, IDB>;
   const size_t smem = (size_t)(KIND == SPLITTERS ? Ly::BYTES_SPL : Ly::BYTES) + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -816,6 +817,13 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
     // 3 CTAs/SM (the deeper prefetch wins for long streams: m8 KO at 2^28 518 vs 499)
     if constexpr (!KV && LOGMP <= 3) {
       if (a.L <= 64ull * (uint64_t)a.sms) return k3v_launch_one<KIND, KV, LOGMP, NT, 2, true, true, false, IDB>(a);
+    }
+    // key-only ONE with 17..32 buckets: tiles of 8192 keys (32 per thread, one key stage, 2 CTAs
+    // per SM) halve the zeroing and scan of the counter matrix per key (the plan passes kpt = 32)
+    if (a.kpt == 32) {
+      if constexpr (!KV && KIND != IDS && LOGMP == 5)
+        return k3v_launch_one<KIND, KV, LOGMP, NT, 1, true, true, false, IDB, 32>(a);
+      return cudaErrorInvalidValue;
     }
     return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true, false, IDB>(a);
   }

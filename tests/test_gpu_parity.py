@@ -103,6 +103,21 @@ def test_ranged_range_edges(kind, m, kv, variant):
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} L={L} n={n} {variant}")
 
 
+@pytest.mark.parametrize("kind,m", [("delta", 32), ("delta", 17), ("splitters", 32), ("lowbits", 32), ("delta", 24)])
+def test_one_k32_edges(kind, m):
+    """Key-only ONE with 17..32 buckets runs tiles of 8192 keys (32 per thread, 2 CTAs/SM):
+    L = ceil(n / 8192) around C = 2 x SMs ranges -- L < C, L = C +- 1, 3C + r, the ragged last
+    tile -- and inputs of one tile or less, 1 launch each."""
+    T = 8192
+    C = 2 * torch.cuda.get_device_properties(0).multi_processor_count
+    sizes = [1, 4095, 4097, 8191, 8192, 8193, 3 * T + 5]
+    for L in (C - 1, C, C + 1, 3 * C + 7):
+        sizes += [L * T, L * T - T + 3]
+    for i, n in enumerate(sizes):
+        case = make_case(kind, m, n, seed=4100 + i, kv=False)
+        _assert_equal(case, _run_case(case, "one"), _expect(case), f"{kind} m={m} n={n} one-k32")
+
+
 @pytest.mark.parametrize("n", [(1 << 26) + 5, 1 << 28])
 @pytest.mark.parametrize("kind,m", [("delta", 2), ("delta", 8), ("lowbits", 16), ("splitters", 16), ("ids", 8),
                                     ("delta", 32), ("ids", 32)])
@@ -531,13 +546,15 @@ def test_max_size_kv_vs_definition():
     assert torch.equal(cursor, exp_off[1:])
 
 
-def test_max_size_ko_properties():
-    """n = 2^32 - 5 keys (the largest n the ABI takes), key-only, m = 8 delta (one ONE launch): the
+@pytest.mark.parametrize("m", [8, 32])
+def test_max_size_ko_properties(m):
+    """n = 2^32 - 5 keys (the largest n the ABI takes), key-only, m = 8 / 32 delta (one ONE launch,
+    tiles of 4096 / 8192 keys; either way > 1024 tiles per CTA, so ONE's counter folding runs): the
     output is the same multiset as the input (order-insensitive 64-bit hashes), its bucket ids never
     decrease, and the offsets are exactly the id boundaries (for key-only output, equal keys are
     interchangeable, so these properties determine the result)."""
     P = _pkg()
-    n, m, delta = (1 << 32) - 5, 8, 1 << 29
+    n, delta = (1 << 32) - 5, (1 << 32) // m
     keys = W.keys_torch(n, 424242, "cuda")
     plan = P.Plan(P.BucketSpec.delta_range(m, delta), n)
     ko, _, off = plan.run(keys)
