@@ -165,9 +165,14 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   const uint32_t beta = 2 * lane + (warp & 1) + 64 * (warp >> 1);
   // (K = 32: the block is the whole swizzled row beta)
   const uint32_t srow = K == 16 ? beta >> 1 : beta, shalf = K == 16 ? beta & 1 : 0;
+  // K = 32: the lanes of a quarter warp read rows 2 apart, which the 128B swizzle maps onto only 4
+  // chunk positions; lanes 4..7 (mod 8) read their chunks rotated by one (step c -> chunk c + 1),
+  // so every 128-bit stage load is conflict-free, and phase 2 rotates the registers back
+  const uint32_t rot = K == 32 ? (lane >> 2) & 1u : 0u;
   uint32_t choff[NCH];  // byte offsets of the block's chunks inside a stage (128B swizzle)
 #pragma unroll
-  for (int c = 0; c < NCH; ++c) choff[c] = srow * 128 + 16 * ((NCH * shalf + c) ^ (srow & 7));
+  for (int c = 0; c < NCH; ++c)
+    choff[c] = srow * 128 + 16 * ((NCH * shalf + ((c + rot) & (NCH - 1))) ^ (srow & 7));
   const uint32_t m = p.m;
   const uint32_t b0 = beta * K;
   // c[j][beta] at shared address ccol + j * RS
@@ -413,8 +418,11 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     if constexpr (FULL) {
       mbar_wait(bar_k + st, ph);
       const uint8_t *sk = sm + Ly::O_SK + st * TB;
+      uint4 raw[NCH];
 #pragma unroll
-      for (int c = 0; c < NCH; ++c) kx[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
+      for (int c = 0; c < NCH; ++c) raw[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) kx[c] = rot ? raw[(c + NCH - 1) & (NCH - 1)] : raw[c];
     } else {
       uint32_t t[K];
 #pragma unroll
@@ -574,6 +582,12 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
         const uint8_t *sv = sm + Ly::O_SV + vst * TB;
 #pragma unroll
         for (int c = 0; c < NCH; ++c) vy[c] = *reinterpret_cast<const uint4 *>(sv + choff[c]);
+        if (rot) {  // (K = 32) back to block order
+          const uint4 last = vy[NCH - 1];
+#pragma unroll
+          for (int c = NCH - 1; c > 0; --c) vy[c] = vy[c - 1];
+          vy[0] = last;
+        }
       } else {
         uint32_t t[K];
 #pragma unroll
