@@ -83,6 +83,11 @@ for _d, _dn in (("binomial", "bin"), ("hot", "hot")):  # skewed north-star workl
         CONFIGS[f"NS{_dn}_{'kv' if _kv else 'ko'}"] = dict(
             desc=f"{'key-value' if _kv else 'key-only'} m=32 delta D=2^27, n=2^28, {_d} buckets", kind="delta",
             m=32, delta=1 << 27, n=1 << 28, kv=_kv, dist=_d, seed=W.SEEDS["C4"])
+for _d, _dn in (("binomial", "bin"), ("hot", "hot")):  # skewed m = 256 workloads (the m > 32 post-scan)
+    for _kv in (False, True):
+        CONFIGS[f"C4{_dn}_{'kv' if _kv else 'ko'}"] = dict(
+            desc=f"{'key-value' if _kv else 'key-only'} m=256 delta D=2^24, n=2^28, {_d} buckets", kind="delta",
+            m=256, delta=1 << 24, n=1 << 28, kv=_kv, dist=_d, seed=W.SEEDS["C4"])
 # precomputed ids (MS_IDS, u8), the fourth bucket kind
 CONFIGS["IDSko"] = dict(desc="key-only m=32 precomputed u8 ids, n=2^28, uniform ids", kind="ids", m=32, n=1 << 28,
                         kv=False, dist="uniform", seed=W.SEEDS["C4"])

@@ -160,7 +160,7 @@ template <int KIND>
 cudaError_t launch_k1(const ms_plan_s *p, const Geometry &g, const uint32_t *keys, const void *ids,
                       uint32_t n, uint32_t *H, uint64_t *zero_ptr, uint32_t zero_words,
                       uint32_t *flag, cudaStream_t s) {
-  const size_t smem = p->spec.m > 32 ? (kMaxM + kWarps * (size_t)p->spec.m) * 4 : k1_smem(p->spec.m, KIND);
+  const size_t smem = p->spec.m > 32 ? (kMaxM + 2 * (size_t)p->spec.m) * 4 : k1_smem(p->spec.m, KIND);
   // one CTA per tile group; SPLITTERS: k1s_prescan on a persistent grid (8 CTAs
   // per SM) so the bin table is built once per CTA
 #define MS_K1(KPT, SUBT)                                                                          \

@@ -132,10 +132,12 @@ k1_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint
   }
 }
 
-// K1 for m > 32: per-warp u32 histograms in shared memory updated with
-// shared-memory atomics (RED.ADD), summed over the tile's warps.  The byte-
-// counter form above zeroes and reduces m * 256 bytes per tile (64 KB at
-// m = 256, 16 B per key); this one touches 8 * m words (2 B per key).
+// K1 for m > 32: one u32 histogram per tile in shared memory, updated by all
+// its warps with shared-memory atomics (round 2: per-warp histograms summed
+// per tile measured 6 % slower, C4 260 vs 243 us).  Bound by the atomics'
+// throughput (about 4 lanes per clock per SM: C4 243 us for 1 GiB of keys,
+// 0.67 of the copy rate).  Byte counters with 64 keys per thread (no atomics,
+// 4 B of counter reduction per key) measured slower still (374 us).
 template <int KIND, int KPT, int SUBT>
 __global__ void __launch_bounds__(kThreads)
 k1a_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uint32_t n,
@@ -143,11 +145,10 @@ k1a_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
             uint64_t *__restrict__ zero_ptr, uint32_t zero_words, uint32_t *__restrict__ err_flag) {
   constexpr int NTS = kThreads / SUBT;   // threads per tile
   constexpr int T = NTS * KPT;           // keys per tile
-  constexpr int WPTILE = kWarps / SUBT;  // warps per tile
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t *spl_s = smem;                // kMaxM words (SPLITTERS)
-  uint32_t *hist = smem + kMaxM;         // [kWarps][m]
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  uint32_t *hist = smem + kMaxM;         // [SUBT][m]: one histogram per tile, all its warps' atomics
+  const uint32_t tid = threadIdx.x, lane = tid & 31;
   const uint32_t h = tid / NTS, tl = tid % NTS;
   const uint64_t tile = (uint64_t)blockIdx.x * SUBT + h;
   const uint64_t base = tile * T;
@@ -163,12 +164,12 @@ k1a_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   }
   pdl_trigger();
   for (uint32_t i = blockIdx.x * kThreads + tid; i < zero_words; i += gridDim.x * kThreads) zero_ptr[i] = 0;
-  for (uint32_t i = tid; i < kWarps * m; i += kThreads) hist[i] = 0;
+  for (uint32_t i = tid; i < SUBT * m; i += kThreads) hist[i] = 0;
   if constexpr (KIND == SPLITTERS) {
     for (uint32_t i = tid; i < (1u << p.logm); i += kThreads) spl_s[i] = p.spl[i];
   }
   __syncthreads();
-  uint32_t *hw = hist + warp * m;
+  uint32_t *hw = hist + h * m;
   uint32_t bad = 0;
   if (full) {
     if constexpr (KIND == IDS) {
@@ -217,9 +218,7 @@ k1a_prescan(const uint32_t *__restrict__ keys, const void *__restrict__ ids, uin
   }
   __syncthreads();
   for (uint32_t b = tl; b < m && tile < L; b += NTS) {
-    uint32_t acc = 0;
-#pragma unroll
-    for (int w = 0; w < WPTILE; ++w) acc += hist[(h * WPTILE + w) * m + b];
+    const uint32_t acc = hist[h * m + b];
     H[(uint64_t)b * L + tile] = acc;
   }
 }

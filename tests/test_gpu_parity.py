@@ -180,7 +180,8 @@ def test_intermediates_H_G_offsets():
     """K1 / K2 intermediates vs the CPU Eq. (2) evaluation with the GPU's tile size T."""
     P = _pkg()
     for kind, m, n in [("delta", 8, 100003), ("splitters", 32, (1 << 20) + 7), ("lowbits", 256, 3 * 8192 + 5),
-                       ("ids", 17, 50000)]:
+                       ("ids", 17, 50000), ("lowbits", 256, 297 * 4096 + 1), ("delta", 100, 299 * 4096 + 77),
+                       ("splitters", 200, 298 * 4096), ("ids", 64, 300 * 4096 + 5)]:
         case = make_case(kind, m, n, seed=m + n, kv=False)
         plan = P.Plan(P.BucketSpec(**case["spec_kw"]), n)
         T, L, _ = plan.geometry(n)
@@ -197,6 +198,22 @@ def test_intermediates_H_G_offsets():
         assert np.array_equal(from_dev(off).astype(np.uint64), eoff)
         ko, _ = plan.postscan(kd, H, ids=idd)
         assert np.array_equal(from_dev(ko), oracle.multisplit(case["ospec"], case["keys"], ids=case["ids"])[0])
+
+
+# m > 32 with 4096-key tiles (from L >= 296; smaller runs use 2048-key tiles): sizes around that
+# boundary, ragged last tiles, every computed kind
+K1B_N = [296 * 4096, 296 * 4096 + 1, 297 * 4096 + 4095, 299 * 4096 + 77]
+
+
+@pytest.mark.parametrize("n", K1B_N)
+@pytest.mark.parametrize("kind,m,seed", [("lowbits", 64, 3), ("lowbits", 256, 0), ("delta", 33, 2),
+                                         ("delta", 100, 1), ("delta", 256, 4), ("splitters", 255, 5),
+                                         ("splitters", 128, 7)])
+def test_parity_m_gt32_4096_tiles(kind, m, seed, n):
+    case = make_case(kind, m, n, seed=seed, kv=seed % 2 == 1)
+    got = _run_case(case)
+    assert got[3].geometry(n)[0] == 4096
+    _assert_equal(case, got, _expect(case), f"{kind} m={m} n={n}")
 
 
 def test_scan_many_chunks():
