@@ -108,7 +108,16 @@ typedef struct ms_plan_s *ms_plan_t;
  * of 8 (tile T = 1024 / 2048 keys; the local reorder then spans fewer warps,
  * the B200 analogue of the paper's NW sweep and of warp- vs block-level
  * reordering); ranged variant, same kinds as
- * MS_ABLATION_DIRECT.  At most one MS_ABLATION_* flag, none with MS_VARIANT_*. */
+ * MS_ABLATION_DIRECT.
+ * MS_ABLATION_BALLOT / MS_ABLATION_WARP: the post-scan of 32 < m <= 256 (Alg. 3
+ * ballot ranks over warp-striped 32-key rounds, ms_k3_warp.cuh) used for any
+ * 2 <= m <= 256, with the block-level reorder of the whole tile (BALLOT,
+ * §5.2.2) or the paper's Warp-level MS (WARP, §5.2.1
+ * every warp reorders only its own 512-key segment, a warp-wide
+ * shuffle scan of its bucket counts giving the positions, and stores its
+ * runs); tile variant, MS_DELTA with m * delta = 2^32 only (else
+ * MS_ERR_UNSUPPORTED).  At most one MS_ABLATION_* flag, none with
+ * MS_VARIANT_*. */
 #define MS_VALIDATE        1u  /* flag precomputed ids >= m on the device; ms_plan_check reports it */
 #define MS_VARIANT_3K      2u
 #define MS_VARIANT_RANGED  4u
@@ -116,6 +125,8 @@ typedef struct ms_plan_s *ms_plan_t;
 #define MS_ABLATION_DIRECT 16u
 #define MS_ABLATION_NW2    32u
 #define MS_ABLATION_NW4    64u
+#define MS_ABLATION_BALLOT 128u
+#define MS_ABLATION_WARP   256u
 
 /* Create a plan for up to max_n elements (max_n < 2^32) on CUDA device
  * `device` (-1: the calling thread's current device; every later call of the

@@ -24,7 +24,7 @@ MS_ERR_BUCKET_RANGE = -8
 
 MS_LOWBITS, MS_DELTA, MS_SPLITTERS, MS_IDS = 0, 1, 2, 3
 MS_VALIDATE, MS_VARIANT_3K, MS_VARIANT_RANGED, MS_VARIANT_ONE, MS_ABLATION_DIRECT = 1, 2, 4, 8, 16
-MS_ABLATION_NW2, MS_ABLATION_NW4 = 32, 64
+MS_ABLATION_NW2, MS_ABLATION_NW4, MS_ABLATION_BALLOT, MS_ABLATION_WARP = 32, 64, 128, 256
 # ms_plan_geometry's variant codes and the kernel launches one ms_run of each enqueues
 VARIANT_TILE, VARIANT_RANGED, VARIANT_ONE, VARIANT_WIDE = 0, 1, 2, 3   # WIDE: m > 256, two passes
 LAUNCHES = {VARIANT_TILE: 3, VARIANT_RANGED: 2, VARIANT_ONE: 1}

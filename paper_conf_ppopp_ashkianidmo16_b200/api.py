@@ -81,14 +81,15 @@ def _check_tensor(t, name):
 
 VARIANT_FLAGS = {None: 0, "3k": _abi.MS_VARIANT_3K, "tile": _abi.MS_VARIANT_3K, "ranged": _abi.MS_VARIANT_RANGED,
                  "one": _abi.MS_VARIANT_ONE, "direct": _abi.MS_ABLATION_DIRECT, "nw2": _abi.MS_ABLATION_NW2,
-                 "nw4": _abi.MS_ABLATION_NW4}
+                 "nw4": _abi.MS_ABLATION_NW4, "ballot": _abi.MS_ABLATION_BALLOT, "warp": _abi.MS_ABLATION_WARP}
 
 
 class Plan:
     """ms_plan_t with a cached device workspace.
 
-    variant: None (chosen per run), "3k"/"tile", "ranged", "one" (MS_VARIANT_*), or
-    "direct" (MS_ABLATION_DIRECT).  device: CUDA ordinal (None = the current device)."""
+    variant: None (chosen per run), "3k"/"tile", "ranged", "one" (MS_VARIANT_*), or an
+    ablation: "direct", "nw2", "nw4", "ballot", "warp" (MS_ABLATION_*, include/ms.h).  device: CUDA
+    ordinal (None = the current device)."""
 
     def __init__(self, spec: BucketSpec, max_n: int, with_values: bool = False, validate: bool = False,
                  variant: str | None = None, device: int | None = None):

@@ -36,6 +36,7 @@ struct ms_plan_s {
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt = 4096
   int forced = -1;      // MS_VARIANT_* flag: the variant every run uses (-1: chosen per run)
   int direct = 0;       // MS_ABLATION_DIRECT: K3 stores keys straight to global, no local reorder
+  int k3w = 0;          // MS_ABLATION_BALLOT (1) / _WARP (2): the ballot K3 for any m, block / warp reorder
   uint32_t k1s_per_sm = 8;  // splitter K1: persistent CTAs per SM (each builds the bin table once)
   int32_t last_launches;
   // m > 256 ("wide"): two stable passes, by the low then the high digit of the id;
@@ -210,10 +211,11 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   a.grid_out = grid_out;
   a.pdl = pdl;
   a.direct = p->direct;
+  a.k3w = p->k3w;
   a.flag = flag;
   a.rowtot = rowtot;
   if (rs) a.rs = *rs;
-  if (p->spec.m <= 32) {  // K3 v2 (ms_k3_v2.cuh), one TU per kind
+  if (p->spec.m <= 32 && !p->k3w) {  // K3 v2 (ms_k3_v2.cuh), one TU per kind
     switch (p->kkind) {
       case LOWBITS: return k3v_launch_lowbits(a);
       case SHIFTC: return k3v_launch_shiftc(a);
@@ -274,7 +276,7 @@ cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, cons
 // 294 vs 283 ONE), >= 16 for m <= 16 and precomputed ids (IDS m=32 KV at 2^25: 236 vs 224),
 // > 64 above (C3 at 2^27: 234 vs 232 ONE vs 224 tile; at 2^25 ONE 212 vs 205) -- ONE below.
 int choose_variant(const ms_plan_s *p, uint64_t L, bool kv) {
-  if (p->spec.m > 32 || p->direct) return V_TILE;
+  if (p->spec.m > 32 || p->direct || p->k3w) return V_TILE;
   if (p->forced >= 0) return p->forced;
   if (!kv) return V_ONE;
   const uint64_t per_sm = p->spec.m <= 8 ? 8 : (p->spec.m <= 16 || p->kkind == IDS) ? 16 : 65;
@@ -550,7 +552,8 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (max_n >= (1ull << 32)) return MS_ERR_INVALID_ARG;
   if (m > (uint32_t)kMaxM) return create_wide(plan, spec, max_n, with_values, flags, device);
   constexpr uint32_t kVariants = MS_VARIANT_3K | MS_VARIANT_RANGED | MS_VARIANT_ONE;
-  constexpr uint32_t kAblations = MS_ABLATION_DIRECT | MS_ABLATION_NW2 | MS_ABLATION_NW4;
+  constexpr uint32_t kAblations =
+      MS_ABLATION_DIRECT | MS_ABLATION_NW2 | MS_ABLATION_NW4 | MS_ABLATION_BALLOT | MS_ABLATION_WARP;
   if (flags & ~(MS_VALIDATE | kVariants | kAblations)) return MS_ERR_INVALID_ARG;
   const uint32_t vf = flags & kVariants, af = flags & kAblations;
   if (vf & (vf - 1)) return MS_ERR_INVALID_ARG;  // at most one variant flag
@@ -598,8 +601,10 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
       break;
     default: return MS_ERR_INVALID_ARG;
   }
-  // the ablations are instantiated for one bucket kind only (DELTA with m * delta = 2^32)
-  if (af && (m > 32 || kkind != SHIFT)) return MS_ERR_UNSUPPORTED;
+  // the ablations are instantiated for one bucket kind only (DELTA with m * delta = 2^32); the
+  // ballot-K3 ablations for 2 <= m <= 256, the others for m <= 32
+  const bool any_m = (af & (MS_ABLATION_BALLOT | MS_ABLATION_WARP)) != 0;
+  if (af && (kkind != SHIFT || (any_m ? m < 2 : m > 32))) return MS_ERR_UNSUPPORTED;
   if (device < -1) return MS_ERR_INVALID_ARG;
   if (device == -1 && cudaGetDevice(&device) != cudaSuccess) {
     cudaGetLastError();
@@ -625,6 +630,7 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   p->forced = (flags & MS_VARIANT_3K) ? V_TILE : (flags & MS_VARIANT_RANGED) ? V_RANGED
             : (flags & MS_VARIANT_ONE) ? V_ONE : -1;
   p->direct = (flags & MS_ABLATION_DIRECT) ? 1 : 0;
+  p->k3w = (flags & MS_ABLATION_BALLOT) ? 1 : (flags & MS_ABLATION_WARP) ? 2 : 0;
   if (flags & (MS_ABLATION_NW2 | MS_ABLATION_NW4)) {  // 2 / 4 warps per K3 CTA: T = 1024 / 2048, ranged
     p->k3nt = (flags & MS_ABLATION_NW2) ? 64u : 128u;
     p->forced = V_RANGED;
@@ -761,7 +767,7 @@ ms_status ms_postscan(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals
 ms_status ms_postscan_scatter(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, const uint32_t *G,
                               uint64_t n, const ms_scatter_target *t, void *ws, size_t ws_bytes, void *stream) {
   if (!p) return MS_ERR_INVALID_ARG;
-  if (p->spec.m > 32 || p->kkind == IDS || p->direct) return MS_ERR_UNSUPPORTED;
+  if (p->spec.m > 32 || p->kkind == IDS || p->direct || p->k3w) return MS_ERR_UNSUPPORTED;
   ms_status st = check_common(p, keys_in, nullptr, n);
   if (st != MS_OK) return st;
   if (!t || t->nranks < 1 || t->nranks > MS_MAX_PEERS) return MS_ERR_INVALID_ARG;

@@ -22,7 +22,7 @@ namespace ms {
 // the tile's bucket starts S_t then give each key its shared-memory slot
 // (Eq. (2) one level down).  Keys (and values) arrive by one TMA
 // bulk copy per array (UBLKCP) on an mbarrier.
-template <int KIND, bool KV, int R, int LOGM, bool FULL>
+template <int KIND, bool KV, int R, int LOGM, bool FULL, bool WL>
 __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
                                         uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
                                         uint64_t base, uint32_t nt, const BucketParams &p,
@@ -122,6 +122,67 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
   }
   __syncthreads();
 
+  if constexpr (WL) {
+    // ---- ablation (MS_ABLATION_WARP): the paper's Warp-level MS (§5.2.1) -- every
+    // warp reorders only its own segment (SEG consecutive keys) and writes its bucket runs:
+    // a warp-wide exclusive scan of the warp's bucket counts (shuffles) gives each key its
+    // position inside the segment, and cnt_w (the warp's tile slot start per bucket, above)
+    // its global position G_j + (slot - S_j).
+    constexpr int BPL = ((1 << LOGM) + 31) / 32;  // buckets per lane
+    uint32_t cw[BPL], st[BPL], sum = 0;
+#pragma unroll
+    for (int b = 0; b < BPL; ++b) {
+      const uint32_t j = lane * BPL + b;
+      cw[b] = st[b] = 0;
+      if (j < m) {
+        st[b] = cnt_w[j];
+        const uint32_t next = warp + 1 < (uint32_t)kWarps ? cnt_s[(warp + 1) * kMaxM + j]
+                              : (j + 1 < m ? cnt_s[j + 1] : nt);  // S_{j+1} = cnt_s[0][j+1]
+        cw[b] = next - st[b];
+      }
+      sum += cw[b];
+    }
+    const uint32_t wincl = warp_incl_scan(sum, lane);
+    const uint32_t wcount = __shfl_sync(0xFFFFFFFFu, wincl, 31);
+    uint32_t ws[BPL], run = wincl - sum;
+#pragma unroll
+    for (int b = 0; b < BPL; ++b) {
+      ws[b] = run;
+      run += cw[b];
+    }
+    __syncthreads();  // every warp has read its successor's cnt_s row
+#pragma unroll
+    for (int b = 0; b < BPL; ++b)
+      if (lane * BPL + b < m) cnt_w[lane * BPL + b] = ws[b];
+    __syncwarp();
+    const uint32_t wbase = warp * SEG;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (FULL || seg0 + r * 32 < nt) {
+        const uint32_t id = pk[r] & 255u;
+        const uint32_t pos = wbase + cnt_w[id] + (pk[r] >> 8);
+        keys_s[pos] = kreg[r];
+        if constexpr (KV) vals_s[pos] = vreg[r];
+        if constexpr (ID8) id8_s[pos] = (uint8_t)id;
+      }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int b = 0; b < BPL; ++b)  // global position of segment slot i = G_j + st_j - S_j + (i - ws_j)
+      if (lane * BPL + b < m) cnt_w[lane * BPL + b] = gD_s[lane * BPL + b] + st[b] - ws[b];
+    __syncwarp();
+    for (uint32_t i = lane; i < wcount; i += 32) {
+      const uint32_t k = keys_s[wbase + i];
+      uint32_t id;
+      if constexpr (ID8) id = id8_s[wbase + i];
+      else id = bucket_of_key<KIND>(k, p, spl_s);
+      const uint32_t dst = cnt_w[id] + i;
+      __stcs(keys_out + dst, k);
+      if constexpr (KV) __stcs(vals_out + dst, vals_s[wbase + i]);
+    }
+    return;
+  }
+
   // ---- local multisplit of the tile into shared memory (in place)
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -153,7 +214,7 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
   }
 }
 
-template <int KIND, bool KV, int R, int LOGM>
+template <int KIND, bool KV, int R, int LOGM, bool WL = false>
 __global__ void __launch_bounds__(kThreads)
 k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
             const void *__restrict__ ids, const uint32_t *__restrict__ G,
@@ -206,10 +267,10 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   __syncthreads();
   if (full) {
     mbar_wait(&bar, 0);
-    k3_tile<KIND, KV, R, LOGM, true>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+    k3_tile<KIND, KV, R, LOGM, true, WL>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
                                spl_s, id8_s, wsum, gcol);
   } else {
-    k3_tile<KIND, KV, R, LOGM, false>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
+    k3_tile<KIND, KV, R, LOGM, false, WL>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
                                 spl_s, id8_s, wsum, gcol);
   }
 }
@@ -220,12 +281,12 @@ inline size_t k3w_smem(int R, bool kv, bool id8) {
   return T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
 }
 
-template <int KIND, bool KV, int R, int LOGM>
+template <int KIND, bool KV, int R, int LOGM, bool WL = false>
 inline cudaError_t k3w_launch_l(const K3pArgs &a) {
   constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC && KIND != SHIFT);
   // ballot ranks (__match_any_sync measured 1.6x slower at m = 256 on B200: MATCH.ANY is
   // ADU-bound)
-  auto k = k3_postscan<KIND, KV, R, LOGM>;
+  auto k = k3_postscan<KIND, KV, R, LOGM, WL>;
   const size_t smem = k3w_smem(R, KV, id8);
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(a.L), dim3(kThreads), smem, a.stream, a.keys, a.vals, a.ids,
@@ -235,6 +296,26 @@ inline cudaError_t k3w_launch_l(const K3pArgs &a) {
 
 template <int KIND, bool KV, int R>
 inline cudaError_t k3w_launch_r(const K3pArgs &a) {
+  if (a.k3w != 0) {  // ablations (MS_ABLATION_BALLOT / _WARP), one-shift bucket kind only, 2 <= m <= 256
+    if constexpr (KIND == SHIFT) {
+      uint32_t l = 1;
+      while ((1u << l) < a.m) ++l;
+      const bool wl = a.k3w == 2;
+#define MS_K3W_ABL(LG) return wl ? k3w_launch_l<KIND, KV, R, LG, true>(a) : k3w_launch_l<KIND, KV, R, LG, false>(a)
+      switch (l) {
+        case 1: MS_K3W_ABL(1);
+        case 2: MS_K3W_ABL(2);
+        case 3: MS_K3W_ABL(3);
+        case 4: MS_K3W_ABL(4);
+        case 5: MS_K3W_ABL(5);
+        case 6: MS_K3W_ABL(6);
+        case 7: MS_K3W_ABL(7);
+        default: MS_K3W_ABL(8);
+      }
+#undef MS_K3W_ABL
+    }
+    return cudaErrorNotSupported;
+  }
   if (a.m <= 64) return k3w_launch_l<KIND, KV, R, 6>(a);
   if (a.m <= 128) return k3w_launch_l<KIND, KV, R, 7>(a);
   return k3w_launch_l<KIND, KV, R, 8>(a);

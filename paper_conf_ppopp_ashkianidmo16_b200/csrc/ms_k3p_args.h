@@ -50,6 +50,8 @@ struct K3pArgs {
   RangeScan rs = {nullptr, nullptr, 0, 0};  // ranged / ONE: the range scan's input (K3's prologue)
   const DistTarget *ds = nullptr;           // fused sharded scatter (K3 v2, tile variant only)
   int direct = 0;                           // ablation: K3 v2 without the local reorder (MS_ABLATION_DIRECT)
+  int k3w = 0;                              // ablation: the ballot K3 (ms_k3_warp.cuh) for any m, block-level (1,
+                                            // MS_ABLATION_BALLOT) or warp-level (2, MS_ABLATION_WARP) reorder
   uint32_t *flag = nullptr;                 // IDS + validation: set to 1 when some id >= m
   const uint32_t *rowtot = nullptr;         // m > 32: G holds row-local scans, term 1 in rowtot[j] (row base)
 };

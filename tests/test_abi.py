@@ -47,7 +47,8 @@ def _create(spec: BucketSpec, max_n=1 << 20, kv=0, flags=0, device=-1):
     (BucketSpec("delta", 8, delta=5), 4 | 8),
     (BucketSpec("delta", 8, delta=5), 2 | 8),
     (BucketSpec("delta", 8, delta=1 << 29), 16 | 2),  # ablation + forced variant
-    (BucketSpec("delta", 8, delta=5), 128),        # unknown flag
+    (BucketSpec("delta", 8, delta=5), 512),        # unknown flag
+    (BucketSpec("delta", 64, delta=1 << 26), 128 | 256),  # two ablations
     (BucketSpec("delta", 8, delta=1 << 29), 32 | 64),  # two ablations
 ])
 def test_plan_create_rejects(spec, flags):
@@ -78,10 +79,21 @@ def test_plan_create_accepts(spec):
     (BucketSpec("ids", 8), 16),
     (BucketSpec("delta", 8, delta=5), 32),         # NW ablations: the same one bucket kind
     (BucketSpec("delta", 64, delta=1 << 26), 64),
+    (BucketSpec("delta", 8, delta=5), 128),        # ballot / warp-level ablations: SHIFT kind, 2 <= m <= 256
+    (BucketSpec("delta", 1, delta=1 << 31), 256),
+    (BucketSpec("lowbits", 64), 256),
 ])
 def test_plan_create_unsupported(spec, flags):
     st, h = _create(spec, flags=flags)
     assert st == _abi.MS_ERR_UNSUPPORTED and not h.value
+
+
+@pytest.mark.parametrize("m", [2, 32, 64, 256])
+@pytest.mark.parametrize("flag", [128, 256])
+def test_ballot_warp_ablations_tile_variant(m, flag):
+    """MS_ABLATION_BALLOT / _WARP are accepted for the SHIFT kind at any 2 <= m <= 256 and run the
+    tile variant (K1 -> K2 -> ballot K3)."""
+    assert _variant(BucketSpec("delta", m, delta=(1 << 32) // m), 1 << 24, False, flags=flag) == _abi.VARIANT_TILE
 
 
 def test_plan_create_device_argument():

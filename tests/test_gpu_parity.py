@@ -21,7 +21,7 @@ def _pkg():
     return P
 
 
-FORCED = {"3k": 0, "tile": 0, "direct": 0, "ranged": 1, "one": 2, "nw2": 1, "nw4": 1}
+FORCED = {"3k": 0, "tile": 0, "direct": 0, "ranged": 1, "one": 2, "nw2": 1, "nw4": 1, "ballot": 0, "warp": 0}
 
 
 def _run_case(case, variant=None, want_offsets=True, expect_variant=None):
@@ -441,6 +441,21 @@ def test_parity_direct_ablation(m):
             case = make_case("delta", m, n, seed=2 * (400 + i), kv=kv)  # even seed: delta = 2^32 / m
             assert case["spec_kw"]["delta"] == (1 << 32) // m
             _assert_equal(case, _run_case(case, "direct"), _expect(case), f"direct m={m} n={n} kv={kv}")
+
+
+@pytest.mark.parametrize("variant", ["ballot", "warp"])
+@pytest.mark.parametrize("m", [2, 8, 16, 32, 64, 128, 256])
+def test_parity_ballot_warp_ablations(variant, m):
+    """The ballot post-scan (Alg. 3 ranks) at any m with block-level (MS_ABLATION_BALLOT) or the
+    paper's warp-level reorder (MS_ABLATION_WARP, §5.2.1: every warp reorders and stores its own
+    512-key segment), bit-exact on ragged sizes (2048- and 4096-key tiles, partial last tiles,
+    partly filled warp segments), uniform and skewed buckets, KO and KV (3 launches)."""
+    for i, n in enumerate([1, 31, 513, 4095, 4097, 100003, 297 * 4096 + 1, (1 << 22) + 3]):
+        for kv in (False, True):
+            dist = ("uniform", "binomial", "hot")[i % 3]
+            case = make_case("delta", m, n, seed=2 * (700 + i), kv=kv, dist=dist)
+            assert case["spec_kw"]["delta"] == (1 << 32) // m  # even seed: the SHIFT kind
+            _assert_equal(case, _run_case(case, variant), _expect(case), f"{variant} m={m} n={n} kv={kv}")
 
 
 # ---------------------------------------------------------------- m > 256 (SURVEY NEXT-3)

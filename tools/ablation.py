@@ -5,10 +5,14 @@ every post-scan method for m in {2, 8, 32}, key-only and key-value, n = 2^25, DE
 equally divide the 32-bit domain (one shift), L2 flushed, CUDA events:
   direct  -- tile variant WITHOUT the local reorder: every key stored from registers straight to
              its global position (MS_ABLATION_DIRECT; the paper's "Direct" method)
-  nw2     -- local reorder over 2 warps (1024-key tiles; MS_ABLATION_NW2, ranged variant): the
-             B200 analogue of the paper's warp-level reordering
+  warp    -- the paper's Warp-level MS: Alg. 3 ballot ranks, every warp reorders and
+             stores its own 512-key segment (MS_ABLATION_WARP, tile variant)
+  ballot  -- the same ballot post-scan with the block-level reorder of the 4096-key tile
+             (MS_ABLATION_BALLOT; the paper's Block-level MS with Alg. 3)
+  nw2     -- blocked-count reorder over 2 warps (1024-key tiles; MS_ABLATION_NW2, ranged variant)
   nw4     -- reorder over 4 warps (2048-key tiles; MS_ABLATION_NW4, ranged)
-  tile    -- block-level reorder over 8 warps (4096-key tiles), K1 -> K2 -> K3 (MS_VARIANT_3K)
+  tile    -- blocked-count block-level reorder over 8 warps (4096-key tiles), K1 -> K2 -> K3
+             (MS_VARIANT_3K; the library's K3 v2)
   ranged  -- the same over CTA ranges, K1r -> K3 (MS_VARIANT_RANGED)
   one     -- the same in one cooperative launch (MS_VARIANT_ONE)
 nw2 / nw4 / ranged together are the NW (warps per CTA) sweep of §6.1.
@@ -25,8 +29,9 @@ import workloads as W  # noqa: E402
 
 steps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
 e = int(sys.argv[2]) if len(sys.argv) > 2 else 25
-modes = ["direct", "nw2", "nw4", "tile", "ranged", "one"]
-variant = {"direct": "direct", "nw2": "nw2", "nw4": "nw4", "tile": "3k", "ranged": "ranged", "one": "one"}
+modes = ["direct", "warp", "ballot", "nw2", "nw4", "tile", "ranged", "one"]
+variant = {"direct": "direct", "warp": "warp", "ballot": "ballot", "nw2": "nw2", "nw4": "nw4", "tile": "3k",
+           "ranged": "ranged", "one": "one"}
 print(f"| m | mode | method | launches | pre-scan ms | scan ms | post-scan ms | total ms (traced) | G keys/s |")
 print("|---|---|---|---|---|---|---|---|---|")
 for m in (2, 8, 32):
