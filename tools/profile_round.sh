@@ -15,10 +15,10 @@ cap() {  # cap CONFIG KERNEL_REGEX
 }
 cap NSko k3v_postscan
 cap NSkv k3v_postscan
-cap NSkv k1_prescan
+cap NSkv k1r_prescan
 cap C4ko k3_postscan
 cap C4ko k1a_prescan
-cap C4ko k2_scan
+cap C4ko k2w_rowscan
 cap C3 k3v_postscan
 cap IDSko k3v_postscan
 ls gpurun_out | grep prof_${TAG}

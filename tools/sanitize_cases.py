@@ -1,6 +1,6 @@
 """Small multisplit cases for compute-sanitizer (memcheck / racecheck / synccheck / initcheck):
 every kernel family once -- ONE (KO, KV, IDS), CTA-range K1r -> K3, tile K1 -> K2 -> K3 for m <= 32
-and m = 256, the Direct ablation, and the fused sharded scatter over virtual ranks -- each checked
+and m = 256, the Direct / NW / ballot / warp-level ablations, and the fused sharded scatter over virtual ranks -- each checked
 against the CPU oracle so a run under the sanitizer is also a parity run.
 
 usage: compute-sanitizer --tool racecheck python tools/sanitize_cases.py [n]"""
@@ -25,11 +25,12 @@ cases = [("delta", 8, False, "one"), ("delta", 8, True, "one"), ("splitters", 32
          ("ids", 32, True, "one"), ("lowbits", 16, True, "ranged"), ("splitters", 32, True, "ranged"),
          ("delta", 32, False, "3k"), ("ids", 5, True, "3k"), ("delta", 256, False, "3k"),
          ("splitters", 200, True, "3k"), ("ids", 100, False, "3k"), ("delta", 256, True, None),
-         ("splitters", 100, False, None), ("delta", 8, False, "nw2"), ("delta", 32, True, "nw4")]
+         ("splitters", 100, False, None), ("delta", 8, False, "nw2"), ("delta", 32, True, "nw4"),
+         ("delta", 32, True, "warp"), ("delta", 256, False, "warp"), ("delta", 8, False, "ballot")]
 fails = 0
 for kind, m, kv, variant in cases:
     # even seeds for the NW ablations: make_case then picks delta = 2^32 / m (the one-shift kind they need)
-    case = make_case(kind, m, n, seed=2 * m if variant in ("nw2", "nw4") else m + 3, kv=kv, dist="binomial")
+    case = make_case(kind, m, n, seed=2 * m if variant in ("nw2", "nw4", "warp", "ballot") else m + 3, kv=kv, dist="binomial")
     plan = P.Plan(P.BucketSpec(**case["spec_kw"]), n, with_values=kv, variant=variant)
     ko, vo, off = plan.run(to_dev(case["keys"]), to_dev(case["vals"]), to_dev(case["ids"]))
     torch.cuda.synchronize()
