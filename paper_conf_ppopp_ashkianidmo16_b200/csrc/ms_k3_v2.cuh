@@ -36,6 +36,10 @@
 
 #include "ms_k3p_args.h"
 
+#ifndef MS_K32_MINM
+#define MS_K32_MINM 9  // key-only ONE with 8192-key tiles from this many buckets
+#endif
+
 namespace ms {
 
 template <int LOGMP, bool KV, int NT, int STAGES, int KPT = 16>
@@ -193,6 +197,13 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
   // ONE, key-only (two stages): phase 1 reads the keys through the TMA stages too (measured
   // better than plain loads: C2 389 vs 371 G keys/s); key-value (one stage): plain coalesced loads
   constexpr bool P1TMA = ONE && !KV && KIND != IDS;
+  // ... and with a single key stage (the 8192-key tiles) phase 1 double-buffers through the reorder
+  // buffer, which phase 2 needs only later: odd phase-1 tiles land there, on the (unused key-only)
+  // value mbarrier, so one tile's load is in flight while the previous one is counted
+#ifndef MS_P1X
+#define MS_P1X 1
+#endif
+  constexpr bool P1X = MS_P1X && P1TMA && STAGES == 1;
   // TMA sequence numbers: ONE keys: [P1TMA: phase 1 forward over the nf full tiles, then] phase 2
   // reverse; ONE values: phase 2 only.  Otherwise sequence = iteration.
   auto seq_tile = [&](uint32_t sq, bool values) -> uint64_t {
@@ -228,6 +239,12 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       if (s < nk) issue(s, false);
       if constexpr (KV) {
         if (s < nv) issue(s, true);
+      }
+    }
+    if constexpr (P1X) {
+      if (nf >= 2) {
+        mbar_arrive_expect_tx(bar_v, TB);
+        tma_load_2d(sm + Ly::O_KS, &tmk, 0, (int)((r0 + 1) * (T / 32)), bar_v);
       }
     }
   }
@@ -292,8 +309,10 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     };
     if constexpr (P1TMA) {
       for (uint32_t sq = 0; sq < nf; ++sq) {
-        mbar_wait(bar_k + sq % STAGES, (sq / STAGES) & 1u);
-        const uint8_t *sk = sm + Ly::O_SK + (sq % STAGES) * TB;
+        const bool odd = P1X && (sq & 1u);
+        if (P1X) mbar_wait(odd ? bar_v : bar_k, (sq >> 1) & 1u);
+        else mbar_wait(bar_k + sq % STAGES, (sq / STAGES) & 1u);
+        const uint8_t *sk = odd ? sm + Ly::O_KS : sm + Ly::O_SK + (sq % STAGES) * TB;
         uint4 kx[NCH];
 #pragma unroll
         for (int c = 0; c < NCH; ++c) kx[c] = *reinterpret_cast<const uint4 *>(sk + choff[c]);
@@ -301,7 +320,19 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
         // the stage may be refilled only once every thread's loads of it have
         // RETURNED (values consumed above), not merely been issued
         __syncthreads();
-        if (tid == 0 && sq + STAGES < 2 * nf) issue(sq + STAGES, false);
+        if constexpr (P1X) {
+          if (tid == 0) {
+            if (sq + 2 < nf) {  // the next tile of this buffer
+              mbar_arrive_expect_tx(odd ? bar_v : bar_k, TB);
+              tma_load_2d(odd ? sm + Ly::O_KS : sm + Ly::O_SK, &tmk, 0, (int)((r0 + sq + 2) * (T / 32)),
+                          odd ? bar_v : bar_k);
+            } else if (!odd) {
+              issue(nf, false);  // phase 2's first tile into the key stage (exactly one of the last two)
+            }
+          }
+        } else {
+          if (tid == 0 && sq + STAGES < 2 * nf) issue(sq + STAGES, false);
+        }
         if ((sq & (FOLDT - 1)) == FOLDT - 1) fold();
       }
     }
@@ -384,7 +415,8 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     // a partial tile, processed first in the reverse walk, has none)
     const uint32_t kq = ONE ? (P1TMA ? nf : 0u) + it - ptail : it, vq = ONE ? it - ptail : it;
     const int st = (int)(kq % STAGES);
-    const uint32_t ph = (kq / STAGES) & 1u;
+    // (P1X: the key mbarrier completed (nf + 1) / 2 phase-1 loads before phase 2's first)
+    const uint32_t ph = P1X ? ((nf + 1) / 2 + kq - nf) & 1u : (kq / STAGES) & 1u;
     const int vst = (int)(vq % STAGES);
     const uint32_t vph = (vq / STAGES) & 1u;
     uint32_t *meta = reinterpret_cast<uint32_t *>(sm + Ly::O_META) + (it & 1) * Ly::MW;
@@ -832,10 +864,10 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
     if constexpr (!KV && LOGMP <= 3) {
       if (a.L <= 64ull * (uint64_t)a.sms) return k3v_launch_one<KIND, KV, LOGMP, NT, 2, true, true, false, IDB>(a);
     }
-    // key-only ONE with 17..32 buckets: tiles of 8192 keys (32 per thread, one key stage, 2 CTAs
+    // key-only ONE with 9..32 buckets: tiles of 8192 keys (32 per thread, one key stage, 2 CTAs
     // per SM) halve the zeroing and scan of the counter matrix per key (the plan passes kpt = 32)
     if (a.kpt == 32) {
-      if constexpr (!KV && KIND != IDS && LOGMP == 5)
+      if constexpr (!KV && KIND != IDS && (1 << LOGMP) >= MS_K32_MINM)
         return k3v_launch_one<KIND, KV, LOGMP, NT, 1, true, true, false, IDB, 32>(a);
       return cudaErrorInvalidValue;
     }

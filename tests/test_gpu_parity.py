@@ -103,15 +103,17 @@ def test_ranged_range_edges(kind, m, kv, variant):
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} L={L} n={n} {variant}")
 
 
-@pytest.mark.parametrize("kind,m", [("delta", 32), ("delta", 17), ("splitters", 32), ("lowbits", 32), ("delta", 24)])
+@pytest.mark.parametrize("kind,m", [("delta", 32), ("delta", 17), ("splitters", 32), ("lowbits", 32), ("delta", 24),
+                                    ("delta", 9), ("lowbits", 16), ("splitters", 12)])
 def test_one_k32_edges(kind, m):
-    """Key-only ONE with 17..32 buckets runs tiles of 8192 keys (32 per thread, 2 CTAs/SM):
-    L = ceil(n / 8192) around C = 2 x SMs ranges -- L < C, L = C +- 1, 3C + r, the ragged last
-    tile -- and inputs of one tile or less, 1 launch each."""
+    """Key-only ONE with 9..32 buckets runs tiles of 8192 keys (32 per thread, 2 CTAs/SM, phase 1
+    double-buffered through the reorder buffer): L = ceil(n / 8192) around C = 2 x SMs ranges --
+    L < C, L = C +- 1, 2C + 1, 3C + r, 5C + 3 (ranges of 1..6 full tiles, odd and even counts),
+    the ragged last tile -- and inputs of one tile or less, 1 launch each."""
     T = 8192
     C = 2 * torch.cuda.get_device_properties(0).multi_processor_count
     sizes = [1, 4095, 4097, 8191, 8192, 8193, 3 * T + 5]
-    for L in (C - 1, C, C + 1, 3 * C + 7):
+    for L in (C - 1, C, C + 1, 2 * C + 1, 3 * C + 7, 5 * C + 3):
         sizes += [L * T, L * T - T + 3]
     for i, n in enumerate(sizes):
         case = make_case(kind, m, n, seed=4100 + i, kv=False)
