@@ -859,7 +859,7 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
     // key-only, 9..32 buckets (computed ids): tiles of 8192 keys, 32 per thread (DESIGN.md §7:
     // half the counter-matrix work per key, phase 1 double-buffered; NSko 440 -> 507, m16 500 ->
     // 526 G keys/s; m <= 8 keeps the 16-key tiles)
-    const bool k32 = vals_in == nullptr && p->spec.m >= MS_K32_MINM && p->kkind != IDS && p->k3nt == 256 && !p->direct;
+    const bool k32 = vals_in == nullptr && p->spec.m >= MS_K32_MINM && (p->kkind != IDS || p->spec.id_bytes == 1) && p->k3nt == 256 && !p->direct;
     const cudaError_t e1 = dispatch_k3(p, k32 ? geometry(p, n, 32) : g, keys_in, vals_in, ids, nullptr, keys_out,
                                        vals_out, (uint32_t)n, flag, s, 2, nullptr, 0, &rs);
     if (e1 == cudaSuccess) {

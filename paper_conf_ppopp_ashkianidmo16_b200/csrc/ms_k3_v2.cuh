@@ -337,7 +337,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
       }
     }
     if constexpr (KIND == IDS) {  // precomputed ids: phase 1 reads only the ids (coalesced 16-byte chunks)
-      constexpr int CH = IDB == 1 ? 1 : NCH;  // 16-byte chunks per thread per tile
+      constexpr int CH = IDB == 1 ? K / 16 : NCH;  // 16-byte chunks per thread per tile
       for (uint32_t sq = 0; sq < nf; ++sq) {
         const uint64_t tb = (r0 + sq) * T;
 #pragma unroll
@@ -395,14 +395,17 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
 
   // one tile; FULL (compile time): all T keys valid, TMA-staged.  The partial
   // tile (at most one, the last of its CTA) is peeled off the loop
-  // MS_IDS with u8 ids: the next full tile's 16 ids of this thread are loaded one tile ahead
+  // MS_IDS with u8 ids: the next full tile's K ids of this thread are loaded one tile ahead
   // (a register double buffer), so their HBM latency overlaps a whole tile instead of stalling the
   // counting pass
-  uint4 idpre = make_uint4(0, 0, 0, 0);
+  uint4 idpre[K / 16] = {};
   auto id_prefetch = [&](uint32_t it) {
     if constexpr (KIND == IDS && IDB == 1) {
-      if (it < iters && tile_of(it) < Lfull)
-        idpre = __ldcs(reinterpret_cast<const uint4 *>(static_cast<const uint8_t *>(ids) + tile_of(it) * T + b0));
+      if (it < iters && tile_of(it) < Lfull) {
+        const uint4 *src = reinterpret_cast<const uint4 *>(static_cast<const uint8_t *>(ids) + tile_of(it) * T + b0);
+#pragma unroll
+        for (int q = 0; q < K / 16; ++q) idpre[q] = __ldcs(src + q);
+      }
     }
   };
   id_prefetch(ONE ? ptail : 0u);  // the first full tile of the walk
@@ -466,7 +469,11 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     uint32_t idk[KEEP_ID ? NCH : 1];    // kept ids, one byte each
     if constexpr (KIND == IDS) {
       if constexpr (FULL && IDB == 1) {
-        idk[0] = clamp4(idpre.x); idk[1] = clamp4(idpre.y); idk[2] = clamp4(idpre.z); idk[3] = clamp4(idpre.w);
+#pragma unroll
+        for (int q = 0; q < K / 16; ++q) {
+          idk[4 * q] = clamp4(idpre[q].x); idk[4 * q + 1] = clamp4(idpre[q].y);
+          idk[4 * q + 2] = clamp4(idpre[q].z); idk[4 * q + 3] = clamp4(idpre[q].w);
+        }
         id_prefetch(it + 1);
       } else if constexpr (FULL) {
         load_ids_full(base + b0, idk, 4);
@@ -867,7 +874,7 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
     // key-only ONE with 9..32 buckets: tiles of 8192 keys (32 per thread, one key stage, 2 CTAs
     // per SM) halve the zeroing and scan of the counter matrix per key (the plan passes kpt = 32)
     if (a.kpt == 32) {
-      if constexpr (!KV && KIND != IDS && (1 << LOGMP) >= MS_K32_MINM)
+      if constexpr (!KV && (KIND != IDS || IDB == 1) && (1 << LOGMP) >= MS_K32_MINM)
         return k3v_launch_one<KIND, KV, LOGMP, NT, 1, true, true, false, IDB, 32>(a);
       return cudaErrorInvalidValue;
     }

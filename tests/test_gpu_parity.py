@@ -104,10 +104,10 @@ def test_ranged_range_edges(kind, m, kv, variant):
 
 
 @pytest.mark.parametrize("kind,m", [("delta", 32), ("delta", 17), ("splitters", 32), ("lowbits", 32), ("delta", 24),
-                                    ("delta", 9), ("lowbits", 16), ("splitters", 12)])
+                                    ("delta", 9), ("lowbits", 16), ("splitters", 12), ("ids", 32), ("ids", 9)])
 def test_one_k32_edges(kind, m):
-    """Key-only ONE with 9..32 buckets runs tiles of 8192 keys (32 per thread, 2 CTAs/SM, phase 1
-    double-buffered through the reorder buffer): L = ceil(n / 8192) around C = 2 x SMs ranges --
+    """Key-only ONE with 9..32 buckets runs tiles of 8192 keys (32 per thread, 2 CTAs/SM; computed
+    ids: phase 1 double-buffered through the reorder buffer; u8 ids: 32 prefetched per thread): L = ceil(n / 8192) around C = 2 x SMs ranges --
     L < C, L = C +- 1, 2C + 1, 3C + r, 5C + 3 (ranges of 1..6 full tiles, odd and even counts),
     the ragged last tile -- and inputs of one tile or less, 1 launch each."""
     T = 8192
