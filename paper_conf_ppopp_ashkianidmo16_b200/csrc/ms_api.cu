@@ -32,7 +32,7 @@ struct ms_plan_s {
   int kkind;  // kernel-level Kind (ms_device.cuh)
   int device;  // CUDA ordinal every call of this plan runs on
   int sms;     // its SM count
-  uint32_t kpt = 16;    // K3 (m <= 32): keys per thread (32 for key-only ONE runs of 9..32 buckets)
+  uint32_t kpt = 16;    // K3 (m <= 32): keys per thread (32 for key-only ONE runs)
   uint32_t k3nt = 256;  // K3 (m <= 32): threads per CTA; tile T = k3nt * kpt = 4096
   int forced = -1;      // MS_VARIANT_* flag: the variant every run uses (-1: chosen per run)
   int direct = 0;       // MS_ABLATION_DIRECT: K3 stores keys straight to global, no local reorder
@@ -54,7 +54,7 @@ struct ms_plan_s {
 };
 
 #ifndef MS_K32_MINM
-#define MS_K32_MINM 9
+#define MS_K32_MINM 2
 #endif
 namespace {
 // returns the 4 events for the next traced run (nullptr when not tracing)
@@ -856,10 +856,13 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
       cudaEventRecord(ev[1], s);
       cudaEventRecord(ev[2], s);
     }
-    // key-only, 9..32 buckets (computed ids): tiles of 8192 keys, 32 per thread (DESIGN.md §7:
-    // half the counter-matrix work per key, phase 1 double-buffered; NSko 440 -> 507, m16 500 ->
-    // 526 G keys/s; m <= 8 keeps the 16-key tiles)
-    const bool k32 = vals_in == nullptr && p->spec.m >= MS_K32_MINM && (p->kkind != IDS || p->spec.id_bytes == 1) && p->k3nt == 256 && !p->direct;
+    // key-only (computed or u8 ids): tiles of 8192 keys, 32 per thread (half the
+    // counter-matrix work per key, phase 1 double-buffered; NSko 440 -> 507, m16 500 -> 526 G
+    // keys/s) for 9..32 buckets, and for m <= 8 above 64 (4096-key) tiles per SM (m8 530 -> 539;
+    // smaller m <= 8 runs keep the two-stage 4-CTA/SM form)
+    const bool k32 = vals_in == nullptr && p->spec.m >= MS_K32_MINM &&
+                     (p->kkind != IDS || p->spec.id_bytes == 1) && p->k3nt == 256 && !p->direct &&
+                     (p->spec.m > 8 || g.L > 64ull * (uint64_t)p->sms);
     const cudaError_t e1 = dispatch_k3(p, k32 ? geometry(p, n, 32) : g, keys_in, vals_in, ids, nullptr, keys_out,
                                        vals_out, (uint32_t)n, flag, s, 2, nullptr, 0, &rs);
     if (e1 == cudaSuccess) {

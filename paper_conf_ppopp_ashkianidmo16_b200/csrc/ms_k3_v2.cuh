@@ -37,7 +37,7 @@
 #include "ms_k3p_args.h"
 
 #ifndef MS_K32_MINM
-#define MS_K32_MINM 9  // key-only ONE with 8192-key tiles from this many buckets
+#define MS_K32_MINM 2  // key-only ONE with 8192-key tiles from this many buckets
 #endif
 
 namespace ms {
@@ -865,18 +865,19 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
     return cudaErrorNotSupported;
   }
   if (a.ranged == 2) {
+    // key-only ONE with 8192-key tiles (32 per thread, one key stage, 2 CTAs per SM): half the
+    // zeroing and scan of the counter matrix per key; ms_run passes kpt = 32 for 9..32 buckets, and
+    // for m <= 8 above 64 (4096-key) tiles per SM
+    if (a.kpt == 32) {
+      if constexpr (!KV && (KIND != IDS || IDB == 1) && (1 << LOGMP) >= MS_K32_MINM)
+        return k3v_launch_one<KIND, KV, LOGMP, NT, 1, true, true, false, IDB, 32>(a);
+      return cudaErrorInvalidValue;
+    }
     // ONE, key-only, m <= 8: up to 64 tiles per SM two key stages at 4 CTAs/SM (more CTAs to share
     // the fixed cost and the tail: C2, n = 2^25, 408 -> 418 G keys/s), above that three stages at
     // 3 CTAs/SM (the deeper prefetch wins for long streams: m8 KO at 2^28 518 vs 499)
     if constexpr (!KV && LOGMP <= 3) {
       if (a.L <= 64ull * (uint64_t)a.sms) return k3v_launch_one<KIND, KV, LOGMP, NT, 2, true, true, false, IDB>(a);
-    }
-    // key-only ONE with 9..32 buckets: tiles of 8192 keys (32 per thread, one key stage, 2 CTAs
-    // per SM) halve the zeroing and scan of the counter matrix per key (the plan passes kpt = 32)
-    if (a.kpt == 32) {
-      if constexpr (!KV && (KIND != IDS || IDB == 1) && (1 << LOGMP) >= MS_K32_MINM)
-        return k3v_launch_one<KIND, KV, LOGMP, NT, 1, true, true, false, IDB, 32>(a);
-      return cudaErrorInvalidValue;
     }
     return k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, true, false, IDB>(a);
   }
