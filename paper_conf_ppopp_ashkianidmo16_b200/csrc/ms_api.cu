@@ -91,7 +91,7 @@ uint64_t delta_magic(uint32_t d) { return ~0ull / d + 1; }
 // keys stay >= 32 keys = 128 B); halved while the grid would not fill two
 // waves of 148 SMs (small n is launch/latency bound, not HBM bound).
 int rounds_for(uint32_t m, uint64_t n, uint32_t kpt) {
-  if (m <= 32) return (int)kpt;  // blocked-rank K3: T = 256 * kpt for every n
+  if (m <= 32 || (kpt == 32 && m <= 64)) return (int)kpt;  // blocked-rank K3: T = 256 * kpt for every n
   int R = 16;
   while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
   return R;
@@ -218,7 +218,7 @@ cudaError_t dispatch_k3(const ms_plan_s *p, const Geometry &g, const uint32_t *k
   a.flag = flag;
   a.rowtot = rowtot;
   if (rs) a.rs = *rs;
-  if (p->spec.m <= 32 && !p->k3w) {  // K3 v2 (ms_k3_v2.cuh), one TU per kind
+  if ((p->spec.m <= 32 || ranged == 2) && !p->k3w) {  // K3 v2 (ms_k3_v2.cuh), one TU per kind
     switch (p->kkind) {
       case LOWBITS: return k3v_launch_lowbits(a);
       case SHIFTC: return k3v_launch_shiftc(a);
@@ -279,7 +279,11 @@ cudaError_t dispatch_k1r(const ms_plan_s *p, const Geometry &g, uint32_t C, cons
 // 294 vs 283 ONE), >= 16 for m <= 16 and precomputed ids (IDS m=32 KV at 2^25: 236 vs 224),
 // > 64 above (C3 at 2^27: 234 vs 232 ONE vs 224 tile; at 2^25 ONE 212 vs 205) -- ONE below.
 int choose_variant(const ms_plan_s *p, uint64_t L, bool kv) {
-  if (p->spec.m > 32 || p->direct || p->k3w) return V_TILE;
+  if (p->direct || p->k3w) return V_TILE;
+  if (p->spec.m > 32) {  // key-only 33..64 buckets (computed or u8 ids): ONE with 8192-key tiles (§7)
+    const bool one = p->spec.m <= 64 && !kv && (p->kkind != IDS || p->spec.id_bytes == 1);
+    return one && p->forced != V_TILE ? V_ONE : V_TILE;
+  }
   if (p->forced >= 0) return p->forced;
   if (!kv) return V_ONE;
   const uint64_t per_sm = p->spec.m <= 8 ? 8 : (p->spec.m <= 16 || p->kkind == IDS) ? 16 : 65;
@@ -562,7 +566,11 @@ ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t m
   if (vf & (vf - 1)) return MS_ERR_INVALID_ARG;  // at most one variant flag
   if (af & (af - 1)) return MS_ERR_INVALID_ARG;  // at most one ablation
   if (af && vf) return MS_ERR_INVALID_ARG;
-  if ((flags & (MS_VARIANT_RANGED | MS_VARIANT_ONE)) && m > 32) return MS_ERR_UNSUPPORTED;
+  if ((flags & MS_VARIANT_RANGED) && m > 32) return MS_ERR_UNSUPPORTED;
+  // ONE above 32 buckets: key-only, m <= 64, computed or u8 ids
+  if ((flags & MS_VARIANT_ONE) && m > 32 &&
+      (m > 64 || with_values || (spec->kind == MS_IDS && spec->id_bytes != 1)))
+    return MS_ERR_UNSUPPORTED;
   BucketParams bp;
   memset(&bp, 0, sizeof(bp));
   int kkind = spec->kind;
@@ -874,7 +882,7 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
     // was forced, clear the launch error and take the two-launch ranged variant (same result)
     if (e1 != cudaErrorCooperativeLaunchTooLarge || p->forced == V_ONE) return MS_ERR_CUDA;
     cudaGetLastError();
-    variant = V_RANGED;
+    variant = p->spec.m > 32 ? V_TILE : V_RANGED;
   }
   if (variant == V_RANGED) {  // K1r -> K3 over C contiguous tile ranges (ms_ranged.cuh); the range
                               // scan runs in K3's prologue

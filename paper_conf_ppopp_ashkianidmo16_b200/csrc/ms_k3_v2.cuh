@@ -67,8 +67,8 @@ struct K3vLayout {
   static constexpr int O_CNT = O_VS + (KV ? KSR * 4 : 0); // counters
   static constexpr int O_META = O_CNT + CNTB;             // [2][MW] words (tile parity)
   static constexpr int O_WS = O_META + 2 * MW * 4;        // warp sums [16]
-  static constexpr int O_TOT = O_WS + 16 * 4;             // ONE: this range's bucket totals [32]
-  static constexpr int O_BAR = (O_TOT + 32 * 4 + 7) & ~7; // mbarriers: keys [STAGES], values [STAGES]
+  static constexpr int O_TOT = O_WS + 16 * 4;             // ONE: this range's bucket totals [max(MP, 32)]
+  static constexpr int O_BAR = (O_TOT + (MP > 32 ? MP : 32) * 4 + 7) & ~7;  // mbarriers: keys, values [STAGES]
   static constexpr int O_SPL = O_BAR + 2 * STAGES * 8;    // SPLITTERS: padded splitters [256] + bin table
   static constexpr int O_TBL = O_SPL + kMaxM * 4;
   static constexpr int BYTES = O_SPL;                     // + 1024 alignment slack at launch
@@ -267,7 +267,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
     // ---- phase 1: this range's bucket counts (private u16 counter columns,
     // folded into tot_s every 32768 / K tiles so that no counter exceeds 32768)
     constexpr uint32_t FOLDT = 32768u / K;
-    if (tid < 32) tot_s[tid] = 0;
+    if (tid < (MP > 32 ? MP : 32)) tot_s[tid] = 0;
     auto zero_cnt = [&]() {
       uint4 *c4 = reinterpret_cast<uint4 *>(cnt);
       for (int idx = tid; idx < Ly::CNTB / 16; idx += NT) c4[idx] = make_uint4(0, 0, 0, 0);
@@ -724,7 +724,7 @@ k3v_postscan(const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CU
         }
       }
     } else {
-      constexpr uint32_t SPB = NT / 32;
+      constexpr uint32_t SPB = NT / (MP > 32 ? MP : 32);  // threads per bucket run
       const uint32_t b = tid / SPB, sub = tid % SPB;
       if (b < m) {
         const uint32_t len = rowS[b + 1] - rowS[b];
@@ -855,6 +855,13 @@ inline cudaError_t k3v_launch_one(const K3pArgs &a) {
 template <int KIND, bool KV, int LOGMP, int IDB>
 inline cudaError_t k3v_launch_n(const K3pArgs &a) {
   constexpr int NT = 256;
+  if constexpr (LOGMP == 6) {  // 33..64 buckets: only the key-only ONE with 8192-key tiles
+    if constexpr (!KV && (KIND != IDS || IDB == 1)) {
+      if (a.ranged == 2 && a.kpt == 32 && a.nt == 256 && !a.direct)
+        return k3v_launch_one<KIND, KV, LOGMP, NT, 1, true, true, false, IDB, 32>(a);
+    }
+    return cudaErrorNotSupported;
+  } else {
   constexpr int STAGES = KV ? 1 : (LOGMP <= 3 ? 3 : 2);  // m <= 8 key-only: 3 stages still fit 3 CTAs/SM
   if (a.nt != 256) {  // ablation (NW sweep): 2 or 4 warps per CTA, ranged variant, one bucket kind
     if constexpr (KIND == SHIFT) {
@@ -887,6 +894,7 @@ inline cudaError_t k3v_launch_n(const K3pArgs &a) {
   }
   return a.ranged ? k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, true, false, false, IDB>(a)
                   : k3v_launch_one<KIND, KV, LOGMP, NT, STAGES, false, false, false, IDB>(a);
+  }
 }
 
 template <int KIND, bool KV, int IDB>
@@ -898,7 +906,8 @@ inline cudaError_t k3v_launch_kv(const K3pArgs &a) {
     case 2: return k3v_launch_n<KIND, KV, 2, IDB>(a);
     case 3: return k3v_launch_n<KIND, KV, 3, IDB>(a);
     case 4: return k3v_launch_n<KIND, KV, 4, IDB>(a);
-    default: return k3v_launch_n<KIND, KV, 5, IDB>(a);
+    case 5: return k3v_launch_n<KIND, KV, 5, IDB>(a);
+    default: return k3v_launch_n<KIND, KV, 6, IDB>(a);
   }
 }
 

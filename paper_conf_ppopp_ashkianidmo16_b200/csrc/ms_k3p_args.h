@@ -83,19 +83,22 @@ inline cudaError_t launch_ex(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 b
 //   GB[c][j] = sum_{i<j} tot_i + pre_j,  offsets[j] = sum_{i<j} tot_i (CTA 0).
 // Thread (s, j) (j = tid mod MP) sums rows s, s + NS, ... of column j, so one
 // warp load covers 32/MP consecutive rows (contiguous words when m = MP).
-// Every thread of the CTA must call it; `red` is 2*NT words of scratch shared
-// memory that nothing else touches until the caller's next __syncthreads().
+// Every thread of the CTA must call it; `red` is 2*NT + 2*(NT/32)*max(MP, 32)
+// words of scratch shared memory that nothing else touches until the caller's
+// next __syncthreads().  m <= 64 (MP = 64: the key-only ONE of 33..64 buckets).
 // Returns GB[c][row] (0 for row >= m).
 template <int NT, int LOGMP>
 __device__ __forceinline__ uint32_t range_base(const RangeScan &rs, uint32_t m, uint32_t c, uint32_t n,
                                                uint32_t *red, uint32_t row) {
   constexpr uint32_t MP = 1u << LOGMP, NS = NT / MP;
+  static_assert(MP <= 64 && NT >= 2 * MP, "range_base: up to 64 buckets");
   const uint32_t tid = threadIdx.x, j = tid & (MP - 1), s = tid >> LOGMP;
   const uint32_t cut = c * rs.k;
+  // red[0 .. MP): per-bucket sums of the rows before `cut` (pre), red[NT .. NT + MP): from `cut` on
   if (MP >= 4 && m == MP) {
     // m a power of two >= 4: 128-bit loads (thread t always reads column group t mod MP/4 of
     // rows t/(MP/4), (t+NT)/(MP/4), ...), lane-shuffle reduction per warp, then the warps' partials
-    constexpr uint32_t Q4 = MP >= 4 ? MP / 4 : 1, NW = NT / 32;
+    constexpr uint32_t Q4 = MP >= 4 ? MP / 4 : 1, NW = NT / 32, WS = MP > 32 ? MP : 32;
     const uint32_t lane = tid & 31, warp = tid >> 5, cg = tid & (Q4 - 1);
     uint32_t pr[4] = {0u, 0u, 0u, 0u}, po[4] = {0u, 0u, 0u, 0u};
     const uint4 *h4 = reinterpret_cast<const uint4 *>(rs.HC);
@@ -119,63 +122,61 @@ __device__ __forceinline__ uint32_t range_base(const RangeScan &rs, uint32_t m, 
         po[e] += __shfl_xor_sync(0xFFFFFFFFu, po[e], off);
       }
     }
+    uint32_t *part = red + 2 * NT;  // [2][NW][WS] the warps' partials
     if (lane < Q4) {
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
-        red[warp * 32 + cg * 4 + e] = pr[e];
-        red[NT + warp * 32 + cg * 4 + e] = po[e];
+        part[warp * WS + cg * 4 + e] = pr[e];
+        part[NW * WS + warp * WS + cg * 4 + e] = po[e];
       }
     }
     __syncthreads();
-    uint32_t pj = 0, qj = 0;
     if (tid < m) {
+      uint32_t pj = 0, qj = 0;
 #pragma unroll
       for (uint32_t w = 0; w < NW; ++w) {
-        pj += red[w * 32 + tid];
-        qj += red[NT + w * 32 + tid];
+        pj += part[w * WS + tid];
+        qj += part[NW * WS + w * WS + tid];
       }
+      red[tid] = pj;
+      red[NT + tid] = qj;
     }
     __syncthreads();
-    if (tid < 32) {
-      const uint32_t tot = pj + qj;  // 0 for tid >= m
-      const uint32_t start = warp_incl_scan(tot, tid) - tot;
-      if (tid < m) red[NT + tid] = start + pj;
-      if (c == 0 && rs.offsets != nullptr) {
-        if (tid < m) rs.offsets[tid] = start;
-        if (tid == 0) rs.offsets[m] = n;
-      }
-    }
-    __syncthreads();
-    return row < m ? red[NT + row] : 0u;
-  }
-  uint32_t pre = 0, post = 0;
-  if (j < m) {
-    const uint32_t *col = rs.HC + j;
+  } else {
+    uint32_t pre = 0, post = 0;
+    if (j < m) {
+      const uint32_t *col = rs.HC + j;
 #pragma unroll 8
-    for (uint32_t r = s; r < rs.R; r += NS) {
-      const uint32_t v = __ldcg(col + (uint64_t)r * m);
-      if (r < cut) pre += v;
-      else post += v;
+      for (uint32_t r = s; r < rs.R; r += NS) {
+        const uint32_t v = __ldcg(col + (uint64_t)r * m);
+        if (r < cut) pre += v;
+        else post += v;
+      }
     }
-  }
-  red[tid] = pre;
-  red[NT + tid] = post;
-  __syncthreads();
-#pragma unroll
-  for (uint32_t d = NS / 2; d >= 1; d >>= 1) {
-    if (s < d) {
-      red[tid] += red[tid + d * MP];
-      red[NT + tid] += red[NT + tid + d * MP];
-    }
+    red[tid] = pre;
+    red[NT + tid] = post;
     __syncthreads();
+#pragma unroll
+    for (uint32_t d = NS / 2; d >= 1; d >>= 1) {
+      if (s < d) {
+        red[tid] += red[tid + d * MP];
+        red[NT + tid] += red[NT + tid + d * MP];
+      }
+      __syncthreads();
+    }
   }
+  // one warp scans the m <= 64 bucket totals, two buckets per lane: bucket start + the pre part
   if (tid < 32) {
-    const uint32_t pj = tid < m ? red[tid] : 0u;
-    const uint32_t tot = tid < m ? pj + red[NT + tid] : 0u;
-    const uint32_t start = warp_incl_scan(tot, tid) - tot;
-    if (tid < m) red[NT + tid] = start + pj;
+    const uint32_t b0 = 2 * tid, b1 = b0 + 1;
+    const uint32_t p0 = b0 < m ? red[b0] : 0u, t0 = b0 < m ? p0 + red[NT + b0] : 0u;
+    const uint32_t p1 = b1 < m ? red[b1] : 0u, t1 = b1 < m ? p1 + red[NT + b1] : 0u;
+    const uint32_t st0 = warp_incl_scan(t0 + t1, tid) - t0 - t1, st1 = st0 + t0;
+    __syncwarp();
+    if (b0 < m) red[NT + b0] = st0 + p0;
+    if (b1 < m) red[NT + b1] = st1 + p1;
     if (c == 0 && rs.offsets != nullptr) {
-      if (tid < m) rs.offsets[tid] = start;
+      if (b0 < m) rs.offsets[b0] = st0;
+      if (b1 < m) rs.offsets[b1] = st1;
       if (tid == 0) rs.offsets[m] = n;
     }
   }

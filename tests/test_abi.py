@@ -72,8 +72,9 @@ def test_plan_create_accepts(spec):
 
 
 @pytest.mark.parametrize("spec,flags", [
-    (BucketSpec("delta", 64, delta=1 << 26), 4),   # ranged / ONE need m <= 32
-    (BucketSpec("delta", 64, delta=1 << 26), 8),
+    (BucketSpec("delta", 64, delta=1 << 26), 4),   # ranged needs m <= 32, ONE m <= 64 key-only
+    (BucketSpec("delta", 128, delta=1 << 25), 8),
+    (BucketSpec("ids", 64, id_bytes=4), 8),        # ONE above 32 buckets: computed or u8 ids
     (BucketSpec("delta", 8, delta=5), 16),         # Direct ablation: DELTA with m * delta = 2^32 only
     (BucketSpec("delta", 64, delta=1 << 26), 16),
     (BucketSpec("ids", 8), 16),
@@ -126,6 +127,13 @@ def test_variant_rule():
     assert _variant(d8, 1 << 28, 1) == RANGED and _variant(d32, 1 << 28, 1) == RANGED
     assert _variant(BucketSpec("ids", 32), 1 << 25, 1) == RANGED and _variant(BucketSpec("ids", 32), 1 << 23, 1) == ONE
     assert _variant(d256, 1 << 20, 0) == T and _variant(d256, 1 << 28, 1) == T
+    d64 = BucketSpec("delta", 64, delta=1 << 26)  # 33..64 buckets: key-only ONE (8192-key tiles), else tile
+    assert _variant(d64, 1 << 28, 0) == ONE and _variant(d64, 1000, 0) == ONE and _variant(d64, 1 << 28, 1) == T
+    assert _variant(BucketSpec("delta", 33, delta=5), 1 << 24, 0) == ONE
+    assert _variant(BucketSpec("ids", 64), 1 << 24, 0) == ONE
+    assert _variant(BucketSpec("ids", 64, id_bytes=4), 1 << 24, 0) == T
+    assert _variant(BucketSpec("delta", 65, delta=5), 1 << 24, 0) == T
+    assert _variant(d64, 1 << 24, 0, 2) == T and _variant(d64, 1 << 24, 0, 8) == ONE
     for flags, want in ((2, TILE), (4, RANGED), (8, ONE)):
         assert _variant(d8, 1 << 28, 1, flags) == want and _variant(d32, 1000, 0, flags) == want
     assert _variant(d8, 1 << 20, 0, 16) == TILE      # the Direct ablation runs the tile variant

@@ -104,9 +104,10 @@ def test_ranged_range_edges(kind, m, kv, variant):
 
 
 @pytest.mark.parametrize("kind,m", [("delta", 32), ("delta", 17), ("splitters", 32), ("lowbits", 32), ("delta", 24),
-                                    ("delta", 9), ("lowbits", 16), ("splitters", 12), ("ids", 32), ("ids", 9)])
+                                    ("delta", 9), ("lowbits", 16), ("splitters", 12), ("ids", 32), ("ids", 9),
+                                    ("delta", 64), ("lowbits", 64), ("splitters", 40), ("ids", 64), ("delta", 33)])
 def test_one_k32_edges(kind, m):
-    """Key-only ONE with 9..32 buckets (and m <= 8 above 64 tiles per SM) runs tiles of 8192 keys (32 per thread, 2 CTAs/SM; computed
+    """Key-only ONE with 9..64 buckets (and m <= 8 above 64 tiles per SM) runs tiles of 8192 keys (32 per thread, 2 CTAs/SM; computed
     ids: phase 1 double-buffered through the reorder buffer; u8 ids: 32 prefetched per thread): L = ceil(n / 8192) around C = 2 x SMs ranges --
     L < C, L = C +- 1, 2C + 1, 3C + r, 5C + 3 (ranges of 1..6 full tiles, odd and even counts),
     the ragged last tile -- and inputs of one tile or less, 1 launch each."""
@@ -165,6 +166,18 @@ def test_parity_distributions(kind, m, dist):
         case = make_case(kind, m, n, seed=7 + m, dist=dist, kv=True)
         for variant in ([None, "3k", "ranged", "one"] if m <= 32 else [None, "3k"]):
             _assert_equal(case, _run_case(case, variant), _expect(case), f"{kind} m={m} {dist} n={n} {variant}")
+
+
+@pytest.mark.parametrize("dist", ["uniform", "binomial", "hot", "one"])
+@pytest.mark.parametrize("kind,m", [("delta", 64), ("splitters", 48), ("ids", 40), ("lowbits", 64)])
+def test_parity_ko_33_64(kind, m, dist):
+    """Key-only 33..64 buckets: ONE with 8192-key tiles (the default) and the forced tile variant
+    (ballot K3), uniform and skewed, ragged sizes up to 3 * 2^22 + 5 keys."""
+    for n in (4097, (1 << 20) + 7, 3 * (1 << 22) + 5):
+        case = make_case(kind, m, n, seed=11 + m, dist=dist, kv=False)
+        for variant in (None, "3k", "one"):
+            _assert_equal(case, _run_case(case, variant, expect_variant=0 if variant == "3k" else 2),
+                          _expect(case), f"{kind} m={m} {dist} n={n} {variant}")
 
 
 @pytest.mark.parametrize("variant", [None, "3k", "ranged", "one"])
