@@ -865,12 +865,10 @@ ms_status ms_run(ms_plan_t p, const uint32_t *keys_in, const uint32_t *vals_in, 
       cudaEventRecord(ev[2], s);
     }
     // key-only (computed or u8 ids): tiles of 8192 keys, 32 per thread (half the
-    // counter-matrix work per key, phase 1 double-buffered; NSko 440 -> 507, m16 500 -> 526 G
-    // keys/s) for 9..32 buckets, and for m <= 8 above 64 (4096-key) tiles per SM (m8 530 -> 539;
-    // smaller m <= 8 runs keep the two-stage 4-CTA/SM form)
+    // counter-matrix work per key, phase 1 double-buffered; NSko 440 -> 507, m16 500 -> 526, C2
+    // 420 -> 440 G keys/s)
     const bool k32 = vals_in == nullptr && p->spec.m >= MS_K32_MINM &&
-                     (p->kkind != IDS || p->spec.id_bytes == 1) && p->k3nt == 256 && !p->direct &&
-                     (p->spec.m > 8 || g.L > 64ull * (uint64_t)p->sms);
+                     (p->kkind != IDS || p->spec.id_bytes == 1) && p->k3nt == 256 && !p->direct;
     const cudaError_t e1 = dispatch_k3(p, k32 ? geometry(p, n, 32) : g, keys_in, vals_in, ids, nullptr, keys_out,
                                        vals_out, (uint32_t)n, flag, s, 2, nullptr, 0, &rs);
     if (e1 == cudaSuccess) {

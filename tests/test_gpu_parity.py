@@ -105,9 +105,10 @@ def test_ranged_range_edges(kind, m, kv, variant):
 
 @pytest.mark.parametrize("kind,m", [("delta", 32), ("delta", 17), ("splitters", 32), ("lowbits", 32), ("delta", 24),
                                     ("delta", 9), ("lowbits", 16), ("splitters", 12), ("ids", 32), ("ids", 9),
-                                    ("delta", 64), ("lowbits", 64), ("splitters", 40), ("ids", 64), ("delta", 33)])
+                                    ("delta", 64), ("lowbits", 64), ("splitters", 40), ("ids", 64), ("delta", 33),
+                                    ("delta", 2), ("lowbits", 8), ("splitters", 5), ("ids", 3)])
 def test_one_k32_edges(kind, m):
-    """Key-only ONE with 9..64 buckets (and m <= 8 above 64 tiles per SM) runs tiles of 8192 keys (32 per thread, 2 CTAs/SM; computed
+    """Key-only ONE with 2..64 buckets runs tiles of 8192 keys (32 per thread, 2 CTAs/SM; computed
     ids: phase 1 double-buffered through the reorder buffer; u8 ids: 32 prefetched per thread): L = ceil(n / 8192) around C = 2 x SMs ranges --
     L < C, L = C +- 1, 2C + 1, 3C + r, 5C + 3 (ranges of 1..6 full tiles, odd and even counts),
     the ragged last tile -- and inputs of one tile or less, 1 launch each."""
@@ -123,8 +124,8 @@ def test_one_k32_edges(kind, m):
 
 @pytest.mark.parametrize("kind,m", [("delta", 2), ("lowbits", 8), ("splitters", 5), ("ids", 4), ("delta", 3)])
 def test_parity_default_large_ko_small_m(kind, m):
-    """Key-only m <= 8 above 64 tiles per SM takes the 8192-key ONE tiles (below: 4096-key tiles
-    with two stages at 4 CTAs/SM): the library's default at n = 2^26 + 5, bit-exact, 1 launch."""
+    """Key-only m <= 8 takes the 8192-key ONE tiles: the library's default at n = 2^26 + 5 (ranges of
+    ~27 tiles), bit-exact, 1 launch."""
     n = (1 << 26) + 5
     case = make_case(kind, m, n, seed=900 + m, kv=False)
     _assert_equal(case, _run_case(case, expect_variant=2), _expect(case), f"{kind} m={m} n={n}")
