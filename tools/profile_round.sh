@@ -21,6 +21,7 @@ cap C4ko k1a_prescan
 cap C4ko k2w_rowscan
 cap C3 k3v_postscan
 cap IDSko k3v_postscan
+cap sweep_m64_ko k3v_postscan
 ls gpurun_out | grep prof_${TAG}
 # summarise on the box (the .ncu-rep files are too large to bring back): text summaries only
 PROF_OUT=gpurun_out python tools/summarize_profiles.py ${TAG} > /dev/null 2>&1
