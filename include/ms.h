@@ -19,16 +19,18 @@
  * two-pass (3); ms_plan_last_launches how many kernels the last ms_run
  * enqueued):
  *   "tile"   subproblems = the L tiles (H, G are m x L words): K1, K2, K3
- *            (the default for 32 < m <= 256);
+ *            (the default for key-value 32 < m <= 256, key-only 64 < m <= 256,
+ *            and key-only u32 ids above 32 buckets);
  *   "ranged" (m <= 32) subproblems = the C <= 1024 contiguous tile ranges of
  *            K3's persistent CTAs: K1 writes per-range histograms (C x k x m),
  *            K3 folds their scan into its prologue and keeps each tile's G_j as
  *            a running sum inside its range (Eq. (2) applied twice): 2 kernels
  *            (the default for key-value runs of >= 8 (m <= 8), >= 16 (m <= 16,
  *            MS_IDS) or > 64 (m <= 32) tiles per SM);
- *   "ONE"    (m <= 32; every other run) the ranged form in ONE cooperative
- *            launch: range counts, grid barrier, range scan, post-scan
- *            (reverse tile walk) -- 1 kernel.  DESIGN.md §7-8;
+ *   "ONE"    (m <= 32 every other run; key-only 33..64 buckets with computed
+ *            or u8 ids) the ranged form in ONE cooperative launch: range
+ *            counts, grid barrier, range scan, post-scan (reverse tile walk)
+ *            -- 1 kernel; key-only runs use 8192-key tiles.  DESIGN.md §7-8;
  *   "two-pass" (m > 256) two stable multisplits by the low and the high digit
  *            of the id, then the offsets from the sorted output (§7b).
  * Every variant computes the same (unique, stable) result.  The MS_VARIANT_*
@@ -97,7 +99,8 @@ typedef struct ms_plan_s *ms_plan_t;
  * MS_VARIANT_* flag makes every run use that one (at most one may be set):
  *   MS_VARIANT_3K      tile variant  K1 -> K2 -> K3     (3 launches, any m)
  *   MS_VARIANT_RANGED  CTA ranges    K1r -> K3          (2 launches, m <= 32)
- *   MS_VARIANT_ONE     cooperative   one kernel         (1 launch,  m <= 32; a
+ *   MS_VARIANT_ONE     cooperative   one kernel         (1 launch,  m <= 32, or
+ *                      key-only m <= 64 with computed or u8 ids; a
  *                      grid that cannot be co-resident fails with MS_ERR_CUDA
  *                      instead of falling back to the ranged variant)
  * MS_ABLATION_DIRECT: the paper's "Direct" post-scan (Table 4):
@@ -135,7 +138,8 @@ typedef struct ms_plan_s *ms_plan_t;
  * MS_LOWBITS, delta >= 1, sorted splitters, id_bytes) and the flags, and
  * precomputes the bucket-function constants.  Returns MS_ERR_INVALID_ARG on a
  * bad spec or flag combination, MS_ERR_UNSUPPORTED for a variant the spec
- * cannot use (m > 32 with MS_VARIANT_RANGED / MS_VARIANT_ONE). */
+ * cannot use (m > 32 with MS_VARIANT_RANGED; MS_VARIANT_ONE with m > 64, or
+ * with m > 32 and values or u32 ids). */
 ms_status ms_plan_create(ms_plan_t *plan, const ms_bucket_spec *spec, uint64_t max_n,
                          int with_values, uint32_t flags, int device);
 
