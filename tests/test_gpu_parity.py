@@ -394,6 +394,33 @@ def test_repeated_runs_same_workspace():
         assert np.array_equal(from_dev(ko), exp[0]) and np.array_equal(from_dev(vo), exp[1])
 
 
+@pytest.mark.parametrize("kind,m,kv,dist", [("delta", 32, False, "uniform"), ("delta", 64, False, "binomial"),
+                                          ("lowbits", 8, False, "hot"), ("ids", 32, False, "uniform"),
+                                          ("splitters", 32, True, "binomial"), ("delta", 16, True, "uniform"),
+                                          ("delta", 256, False, "uniform")])
+def test_repeat_stress(kind, m, kv, dist):
+    """Race canary (compute-sanitizer was closed on the pool for the round's last kernel changes):
+    1000 back-to-back runs of the default path on one workspace -- the mbarrier / TMA stage reuse,
+    the double-buffered phase 1, the grid barrier and the bulk-store drain all cycle many times per
+    run at this size (~7 tiles per persistent CTA, an odd partial last tile) -- every output compared
+    element-wise on the device with the oracle's."""
+    P = _pkg()
+    n = 296 * 8192 * 3 + 4097 if not kv else 296 * 4096 * 7 + 4097
+    case = make_case(kind, m, n, seed=31 + m, kv=kv, dist=dist)
+    plan = P.Plan(P.BucketSpec(**case["spec_kw"]), n, with_values=kv)
+    kd, vd, idd = to_dev(case["keys"]), to_dev(case["vals"]), to_dev(case["ids"])
+    eko, evo, eoff = _expect(case)
+    ek, ev = to_dev(eko), to_dev(evo)
+    eo = torch.as_tensor(eoff.astype(np.int64), device="cuda")
+    bad = 0
+    for _ in range(1000):
+        ko, vo, off = plan.run(kd, vd, idd)
+        bad += int(not torch.equal(ko, ek)) + int(kv and not torch.equal(vo, ev)) + \
+            int(not torch.equal(off.to(torch.int64) & 0xFFFFFFFF, eo))
+    torch.cuda.synchronize()
+    assert bad == 0, f"{bad} mismatching outputs in 1000 runs"
+
+
 @pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
 @pytest.mark.parametrize("kind,m", [("lowbits", 2), ("delta", 8), ("splitters", 32), ("delta", 5), ("lowbits", 1)])
 def test_fused_scatter_virtual_ranks(P, kind, m):
