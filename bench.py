@@ -101,7 +101,8 @@ CONFIGS["C5s"] = dict(CONFIGS["C5"], n=1 << 26, desc=CONFIGS["C5"]["desc"].repla
 
 DEFAULT = "NSko"      # N = 1 headline
 DEFAULT_DIST = "C5"   # N > 1 headline
-EXTRA_DEFAULT = ",".join(["NSkv", "NSbin_ko", "NShot_ko", "NSbin_kv", "NShot_kv", "C4ko", "C4kv", "C3", "C3bin",
+EXTRA_DEFAULT = ",".join(["NSkv", "NSbin_ko", "NShot_ko", "NSbin_kv", "NShot_kv", "C4ko", "C4kv", "C4bin_ko",
+                          "C4hot_ko", "C3", "C3bin",
                           "C3hot", "C2", "C2far", "C1", "IDSko", "IDSkv"] +
                          [f"sweep_m{m}_{t}" for t in ("ko", "kv") for m in (2, 4, 8, 16, 64, 128)] +
                          [f"wide_m{m}_{t}" for t in ("ko", "kv") for m in (512, 4096, 65536)])
