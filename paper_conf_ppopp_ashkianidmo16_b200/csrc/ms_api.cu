@@ -87,12 +87,15 @@ uint32_t ceil_log2(uint32_t m) {
 // Kurz: exact when the magic has >= 32 + log2(delta) fractional bits).
 uint64_t delta_magic(uint32_t d) { return ~0ull / d + 1; }
 
-// Rounds per warp R (tile T = 256 R): 16 for m <= 32, 32 above (runs of T/m
-// keys stay >= 32 keys = 128 B); halved while the grid would not fill two
-// waves of 148 SMs (small n is launch/latency bound, not HBM bound).
-int rounds_for(uint32_t m, uint64_t n, uint32_t kpt) {
+// Rounds per warp R (subproblem T = 256 R keys): kpt for the blocked-rank K3 (m <= 32, and the
+// key-only ONE up to 64 buckets); for the ballot K3 of m > 32, 32 on key-only plans (8192-key
+// subproblems reordered as two 4096-key windows per CTA: half the H / G words and K1 / K2 work,
+// C4ko 247 -> 259 G keys/s) and 16 on key-value plans (the second window's serialised load costs
+// more there: C4kv 177 -> 155) -- halved while the grid would not fill two waves of 148 SMs (small
+// n is launch / latency bound, not HBM bound).
+int rounds_for(uint32_t m, uint64_t n, uint32_t kpt, bool kv_plan) {
   if (m <= 32 || (kpt == 32 && m <= 64)) return (int)kpt;  // blocked-rank K3: T = 256 * kpt for every n
-  int R = 16;
+  int R = kv_plan ? 16 : 32;
   while (R > 8 && (n + 256ull * R - 1) / (256ull * R) < 2 * 148) R >>= 1;
   return R;
 }
@@ -109,7 +112,7 @@ struct Geometry {
 
 Geometry geometry(const ms_plan_s *p, uint64_t n, uint32_t kpt = 0) {
   Geometry g{};
-  g.R = rounds_for(p->spec.m, n, (kpt ? kpt : p->kpt) * p->k3nt / 256);
+  g.R = rounds_for(p->spec.m, n, (kpt ? kpt : p->kpt) * p->k3nt / 256, p->kv != 0);
   g.T = 256u * g.R;
   g.L = (n + g.T - 1) / g.T;
   g.hg_words = (uint64_t)p->spec.m * g.L;

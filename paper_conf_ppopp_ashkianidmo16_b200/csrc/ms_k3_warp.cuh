@@ -23,7 +23,7 @@ namespace ms {
 // (Eq. (2) one level down).  Keys (and values) arrive by one TMA
 // bulk copy per array (UBLKCP) on an mbarrier.
 template <int KIND, bool KV, int R, int LOGM, bool FULL, bool WL>
-__device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
+__device__ __forceinline__ uint32_t k3_tile(const uint32_t *__restrict__ vals_g, const void *__restrict__ ids,
                                         uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out,
                                         uint64_t base, uint32_t nt, const BucketParams &p,
                                         uint32_t *keys_s, uint32_t *vals_s, uint32_t *cnt_s,
@@ -180,7 +180,7 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
       __stcs(keys_out + dst, k);
       if constexpr (KV) __stcs(vals_out + dst, vals_s[wbase + i]);
     }
-    return;
+    return tot;
   }
 
   // ---- local multisplit of the tile into shared memory (in place)
@@ -212,10 +212,16 @@ __device__ __forceinline__ void k3_tile(const uint32_t *__restrict__ vals_g, con
   } else {
     for (uint32_t i = tid; i < nt; i += kThreads) store(i);
   }
+  return tot;  // this tile's count of bucket tid (tid < m)
 }
 
-template <int KIND, bool KV, int R, int LOGM, bool WL = false>
-__global__ void __launch_bounds__(kThreads)
+// TPC reorder windows of T keys per subproblem (Eq. (2)'s column of G): with TPC = 2 the
+// subproblems are 8192 keys (half the H / G words, K1 and K2 work) while the local reorder keeps
+// 4096-key windows; the CTA walks its windows in order with a running G (the first window's
+// bucket counts added before the second).  Key-only: both windows' TMA loads are issued up front
+// (two buffers); key-value: one buffer, the second window loaded after the first has left.
+template <int KIND, bool KV, int R, int LOGM, bool WL = false, int TPC = 1>
+__global__ void __launch_bounds__(kThreads, KV ? 3 : 4)  // 4 / 3 CTAs per SM (64 / 85 registers)
 k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals,
             const void *__restrict__ ids, const uint32_t *__restrict__ G,
             uint32_t *__restrict__ keys_out, uint32_t *__restrict__ vals_out, uint32_t n,
@@ -223,85 +229,107 @@ k3_postscan(const uint32_t *__restrict__ keys, const uint32_t *__restrict__ vals
   // G: the full Eq. (2) terms 1+2 (K2 = k2_scan), or -- rowbase != nullptr (K2 = k2w_rowscan) --
   // term 2 only, row by row, with term 1 in rowbase[j]
   constexpr int T = kThreads * R;
+  constexpr int NB = (TPC > 1 && !KV) ? TPC : 1;  // window buffers
   extern __shared__ __align__(128) uint8_t smem_raw[];
-  uint32_t *keys_s = reinterpret_cast<uint32_t *>(smem_raw);
-  uint32_t *vals_s = keys_s + T;
+  uint32_t *keys_s0 = reinterpret_cast<uint32_t *>(smem_raw);  // [NB][T]
+  uint32_t *vals_s = keys_s0 + NB * T;
   uint32_t *cnt_s = vals_s + (KV ? T : 0);     // [8][256] per-warp counters
   uint32_t *gD_s = cnt_s + kWarps * kMaxM;     // [256] G[j][tile] - S_t[j]
   uint32_t *spl_s = gD_s + kMaxM;              // [256] padded splitters
   uint8_t *id8_s = reinterpret_cast<uint8_t *>(spl_s + kMaxM);  // [T]
-  __shared__ __align__(8) uint64_t bar;
+  __shared__ __align__(8) uint64_t bar[TPC];
   __shared__ uint32_t wsum[kWarps];
 
   const uint32_t tid = threadIdx.x;
   const uint32_t tile = blockIdx.x;
-  const uint64_t base = (uint64_t)tile * T;
-  const uint32_t nt = (uint32_t)umin64(T, n - base);
-  const bool full = (nt == T);
   const uint32_t m = p.m;
-
-  if (full) {
-    if (tid == 0) {
-      mbar_init(&bar, 1);
-      fence_mbar_init();
-      mbar_arrive_expect_tx(&bar, (KV ? 2u : 1u) * T * 4u);
-      bulk_g2s(keys_s, keys + base, T * 4u, &bar);
-      if constexpr (KV) bulk_g2s(vals_s, vals + base, T * 4u, &bar);
+  auto wbase = [&](int w) -> uint64_t { return ((uint64_t)tile * TPC + w) * T; };
+  auto wnt = [&](int w) -> uint32_t { return wbase(w) < n ? (uint32_t)umin64(T, n - wbase(w)) : 0u; };
+  auto load = [&](int w, uint32_t *ks) {  // window w into ks (+ vals_s): TMA when full, else by hand
+    const uint64_t base = wbase(w);
+    const uint32_t nt = wnt(w);
+    if (nt == T) {
+      if (tid == 0) {
+        mbar_arrive_expect_tx(&bar[w], (KV ? 2u : 1u) * T * 4u);
+        bulk_g2s(ks, keys + base, T * 4u, &bar[w]);
+        if constexpr (KV) bulk_g2s(vals_s, vals + base, T * 4u, &bar[w]);
+      }
+    } else {
+      for (uint32_t i = tid; i < nt; i += kThreads) {
+        ks[i] = keys[base + i];
+        if constexpr (KV) vals_s[i] = vals[base + i];
+      }
     }
-  } else {
-    for (uint32_t i = tid; i < nt; i += kThreads) {
-      keys_s[i] = keys[base + i];
-      if constexpr (KV) vals_s[i] = vals[base + i];
-    }
+  };
+  if (tid == 0) {  // (thread 0 also issues the TMA loads: no barrier needed before them)
+#pragma unroll
+    for (int w = 0; w < TPC; ++w) mbar_init(&bar[w], 1);
+    fence_mbar_init();
+  }
+  load(0, keys_s0);
+  if constexpr (NB > 1) {
+#pragma unroll
+    for (int w = 1; w < TPC; ++w) load(w, keys_s0 + w * T);
   }
   // per-bucket setup while the copy is in flight
   uint32_t gcol = 0;
   pdl_wait();  // K2's G is complete (the tile's TMA load above is already in flight)
   if (tid < m) gcol = __ldg(G + (uint64_t)tid * L + tile);
   if (rowbase != nullptr && tid < m) gcol += __ldg(rowbase + tid);
-#pragma unroll
-  for (int w = 0; w < kWarps; ++w) cnt_s[w * kMaxM + tid] = 0;  // kThreads == kMaxM
   if constexpr (KIND == SPLITTERS) {
     if (tid < (1u << p.logm)) spl_s[tid] = p.spl[tid];
   }
-  __syncthreads();
-  if (full) {
-    mbar_wait(&bar, 0);
-    k3_tile<KIND, KV, R, LOGM, true, WL>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
-                               spl_s, id8_s, wsum, gcol);
-  } else {
-    k3_tile<KIND, KV, R, LOGM, false, WL>(vals, ids, keys_out, vals_out, base, nt, p, keys_s, vals_s, cnt_s, gD_s,
-                                spl_s, id8_s, wsum, gcol);
+#pragma unroll 1
+  for (int w = 0; w < TPC; ++w) {
+    const uint32_t nt = wnt(w);
+    if (nt == 0) break;
+    uint32_t *keys_s = keys_s0 + (NB > 1 ? w * T : 0);
+    if (NB == 1 && w > 0) load(w, keys_s);  // (the previous window's stores have read the buffer)
+#pragma unroll
+    for (int q = 0; q < kWarps; ++q) cnt_s[q * kMaxM + tid] = 0;  // kThreads == kMaxM
+    __syncthreads();
+    uint32_t tot;
+    if (nt == T) {
+      mbar_wait(&bar[w], 0);
+      tot = k3_tile<KIND, KV, R, LOGM, true, WL>(vals, ids, keys_out, vals_out, wbase(w), nt, p, keys_s, vals_s,
+                                                 cnt_s, gD_s, spl_s, id8_s, wsum, gcol);
+    } else {
+      tot = k3_tile<KIND, KV, R, LOGM, false, WL>(vals, ids, keys_out, vals_out, wbase(w), nt, p, keys_s, vals_s,
+                                                  cnt_s, gD_s, spl_s, id8_s, wsum, gcol);
+    }
+    gcol += tot;  // the next window's bucket starts (running G)
+    if (TPC > 1) __syncthreads();  // cnt_s / gD_s / id8_s / the buffers are reused by the next window
   }
 }
 
 // ------------------------------------------------------------------ host launcher (m > 32)
-inline size_t k3w_smem(int R, bool kv, bool id8) {
+inline size_t k3w_smem(int R, bool kv, bool id8, int nb = 1) {
   const size_t T = 256u * R;
-  return T * 4 * (kv ? 2 : 1) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
+  return T * 4 * (kv ? 2 : nb) + (kWarps * kMaxM + 2 * kMaxM) * 4 + (id8 ? T : 0);
 }
 
-template <int KIND, bool KV, int R, int LOGM, bool WL = false>
+template <int KIND, bool KV, int R, int LOGM, bool WL = false, int TPC = 1>
 inline cudaError_t k3w_launch_l(const K3pArgs &a) {
   constexpr bool id8 = (KIND != LOWBITS && KIND != SHIFTC && KIND != SHIFT);
   // ballot ranks (__match_any_sync measured 1.6x slower at m = 256 on B200: MATCH.ANY is
   // ADU-bound)
-  auto k = k3_postscan<KIND, KV, R, LOGM, WL>;
-  const size_t smem = k3w_smem(R, KV, id8);
+  auto k = k3_postscan<KIND, KV, R, LOGM, WL, TPC>;
+  const size_t smem = k3w_smem(R, KV, id8, (TPC > 1 && !KV) ? TPC : 1);
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   const cudaError_t e = launch_ex(a.pdl != 0, k, dim3(a.L), dim3(kThreads), smem, a.stream, a.keys, a.vals, a.ids,
                                   a.G, a.keys_out, a.vals_out, a.n, a.L, *a.bp, a.rowtot);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
-template <int KIND, bool KV, int R>
+template <int KIND, bool KV, int R, int TPC = 1>
 inline cudaError_t k3w_launch_r(const K3pArgs &a) {
   if (a.k3w != 0) {  // ablations (MS_ABLATION_BALLOT / _WARP), one-shift bucket kind only, 2 <= m <= 256
     if constexpr (KIND == SHIFT) {
       uint32_t l = 1;
       while ((1u << l) < a.m) ++l;
       const bool wl = a.k3w == 2;
-#define MS_K3W_ABL(LG) return wl ? k3w_launch_l<KIND, KV, R, LG, true>(a) : k3w_launch_l<KIND, KV, R, LG, false>(a)
+#define MS_K3W_ABL(LG) \
+  return wl ? k3w_launch_l<KIND, KV, R, LG, true, TPC>(a) : k3w_launch_l<KIND, KV, R, LG, false, TPC>(a)
       switch (l) {
         case 1: MS_K3W_ABL(1);
         case 2: MS_K3W_ABL(2);
@@ -316,14 +344,16 @@ inline cudaError_t k3w_launch_r(const K3pArgs &a) {
     }
     return cudaErrorNotSupported;
   }
-  if (a.m <= 64) return k3w_launch_l<KIND, KV, R, 6>(a);
-  if (a.m <= 128) return k3w_launch_l<KIND, KV, R, 7>(a);
-  return k3w_launch_l<KIND, KV, R, 8>(a);
+  if (a.m <= 64) return k3w_launch_l<KIND, KV, R, 6, false, TPC>(a);
+  if (a.m <= 128) return k3w_launch_l<KIND, KV, R, 7, false, TPC>(a);
+  return k3w_launch_l<KIND, KV, R, 8, false, TPC>(a);
 }
 
 template <int KIND>
 inline cudaError_t k3w_launch(const K3pArgs &a) {
   if (a.kpt == 8) return a.vals ? k3w_launch_r<KIND, true, 8>(a) : k3w_launch_r<KIND, false, 8>(a);
+  // 8192-key subproblems (kpt = 32): two 4096-key reorder windows per CTA
+  if (a.kpt == 32) return a.vals ? k3w_launch_r<KIND, true, 16, 2>(a) : k3w_launch_r<KIND, false, 16, 2>(a);
   return a.vals ? k3w_launch_r<KIND, true, 16>(a) : k3w_launch_r<KIND, false, 16>(a);
 }
 

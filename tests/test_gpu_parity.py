@@ -206,7 +206,8 @@ def test_intermediates_H_G_offsets():
     P = _pkg()
     for kind, m, n in [("delta", 8, 100003), ("splitters", 32, (1 << 20) + 7), ("lowbits", 256, 3 * 8192 + 5),
                        ("ids", 17, 50000), ("lowbits", 256, 297 * 4096 + 1), ("delta", 100, 299 * 4096 + 77),
-                       ("splitters", 200, 298 * 4096), ("ids", 64, 300 * 4096 + 5)]:
+                       ("splitters", 200, 298 * 4096), ("ids", 64, 300 * 4096 + 5),
+                       ("delta", 256, 299 * 8192 + 4097), ("lowbits", 128, 297 * 8192)]:
         case = make_case(kind, m, n, seed=m + n, kv=False)
         plan = P.Plan(P.BucketSpec(**case["spec_kw"]), n)
         T, L, _ = plan.geometry(n)
@@ -225,9 +226,11 @@ def test_intermediates_H_G_offsets():
         assert np.array_equal(from_dev(ko), oracle.multisplit(case["ospec"], case["keys"], ids=case["ids"])[0])
 
 
-# m > 32 with 4096-key tiles (from L >= 296; smaller runs use 2048-key tiles): sizes around that
-# boundary, ragged last tiles, every computed kind
-K1B_N = [296 * 4096, 296 * 4096 + 1, 297 * 4096 + 4095, 299 * 4096 + 77]
+# m > 32: 2048-key subproblems below 296 x 4096 keys, 4096-key up to 296 x 8192, and on key-only plans
+# 8192-key ones above (reordered as two 4096-key windows per CTA with a running G): sizes around both
+# boundaries, ragged last subproblems (one full window + a partial one, a partial first window only)
+K1B_N = [296 * 4096, 296 * 4096 + 1, 297 * 4096 + 4095, 299 * 4096 + 77,
+         296 * 8192, 296 * 8192 + 1, 297 * 8192 + 4095, 299 * 8192 + 4097, 300 * 8192 + 77]
 
 
 @pytest.mark.parametrize("n", K1B_N)
@@ -237,7 +240,7 @@ K1B_N = [296 * 4096, 296 * 4096 + 1, 297 * 4096 + 4095, 299 * 4096 + 77]
 def test_parity_m_gt32_4096_tiles(kind, m, seed, n):
     case = make_case(kind, m, n, seed=seed, kv=seed % 2 == 1)
     got = _run_case(case)
-    assert got[3].geometry(n)[0] == 4096
+    assert got[3].geometry(n)[0] == (8192 if n >= 296 * 8192 and seed % 2 == 0 else 4096)  # key-value: 4096
     _assert_equal(case, got, _expect(case), f"{kind} m={m} n={n}")
 
 
